@@ -1,0 +1,349 @@
+"""Pins for the CPU oracle (tests/ only; no GPU).
+
+Each test pins an oracle function to something fixed OUTSIDE the oracle: a
+value printed in a textbook/table (tests/golden/, cited there), a closed form
+derived independently of the oracle's code, a physical invariant, a
+calculus fact, or an independent implementation (numpy BLAS, Python ints,
+math.fsum). Chosen so that a dropped term, wrong sign/index or transposed
+operand in lime_oracle.c fails at least one of them.
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_pldi_dubachcrbf12_b200 import inputs
+from testutil import golden as _golden
+
+
+# =========================================================== N-Body
+# oracle_nbody_accel: PAPER.md L106-114, L156-158; readings R1-R3
+
+def test_nbody_single_body_is_zero():
+    b = np.array([[0.3, -0.2, 0.1, 1.0]], dtype=np.float32)
+    a = oracle.nbody_accel(b, 1e-4)
+    assert np.all(a == 0.0)  # self term contributes exactly 0
+
+
+def test_nbody_two_body_newton_far_field_and_direction():
+    # Newton: |a_0| = G m_1 / d^2 directed toward body 1 (eps -> 0 limit).
+    for d, m1 in [(1.0, 0.5), (2.0, 0.25), (0.5, 1.0)]:
+        b = np.array([[0, 0, 0, 0.125], [0, d, 0, m1]], dtype=np.float32)
+        a = oracle.nbody_accel(b, 1e-12)
+        assert a[0, 1] > 0 and a[1, 1] < 0            # attraction, not repulsion
+        assert abs(a[0, 1] - m1 / d**2) <= 1e-9 * m1 / d**2
+        assert abs(a[1, 1] + 0.125 / d**2) <= 1e-9 * 0.125 / d**2
+        assert a[0, 0] == 0 and a[0, 2] == 0          # no cross-axis leakage
+
+
+def test_nbody_third_law_pair():
+    b = np.array([[0.1, 0.2, -0.3, 0.75], [-0.4, 0.5, 0.6, 0.25]], dtype=np.float32)
+    a = oracle.nbody_accel(b, 1e-4)
+    np.testing.assert_allclose(0.75 * a[0], -0.25 * a[1], rtol=1e-14, atol=0)
+
+
+def test_nbody_plummer_softening_peak():
+    # Calculus fact for Plummer softening: d/dd [d (d^2+e^2)^(-3/2)] = 0 at d = e/sqrt2,
+    # with peak value m * 2 / (3 sqrt3 e^2). Pins the exponent 3/2 and where eps2 enters.
+    eps2 = np.float32(0.01)
+    e = math.sqrt(float(eps2))
+    ds = np.linspace(0.0, 4 * e, 4001)
+    mags = []
+    for d in ds:
+        b = np.array([[0, 0, 0, 1.0], [d, 0, 0, 1.0]], dtype=np.float32)
+        mags.append(oracle.nbody_accel(b, eps2)[0, 0])
+    mags = np.array(mags)
+    dstar = ds[np.argmax(mags)]
+    assert abs(dstar - e / math.sqrt(2)) <= 2 * (ds[1] - ds[0])
+    assert abs(mags.max() - 2.0 / (3.0 * math.sqrt(3.0) * float(eps2))) <= 1e-5 * mags.max()
+
+
+def test_nbody_cube_center_cancels():
+    corners = [(x, y, z) for x in (-1, 1) for y in (-1, 1) for z in (-1, 1)]
+    b = np.array([[*c, 0.5] for c in corners] + [[0, 0, 0, 2.0]], dtype=np.float32)
+    a, A = oracle.nbody_accel(b, 1e-4, with_mag=True)
+    assert np.linalg.norm(a[8]) <= 1e-12 * A[8]
+    # each corner is pulled toward the centre along its diagonal
+    for k, c in enumerate(corners):
+        assert np.dot(a[k], np.array(c, dtype=float)) < 0
+
+
+def test_nbody_regular_polygon_closed_form():
+    # k equal masses on a circle of radius R: by symmetry a_0 is radial (toward the centre) with
+    # |a| = m * sum_{q=1}^{k-1} 2R sin^2(pi q/k) / ((2R sin(pi q/k))^2 + eps2)^{3/2}.
+    k, R, m, eps2 = 12, 0.75, 0.5, np.float32(1e-3)
+    th = 2 * np.pi * np.arange(k) / k
+    b = np.zeros((k, 4), dtype=np.float32)
+    b[:, 0] = R * np.cos(th)
+    b[:, 1] = R * np.sin(th)
+    b[:, 3] = m
+    a = oracle.nbody_accel(b, eps2)
+    # closed form uses the fp32-rounded positions' radius
+    Rf = float(np.hypot(b[0, 0], b[0, 1]))
+    q = np.arange(1, k)
+    s = np.sin(np.pi * q / k)
+    ref = m * np.sum(2 * Rf * s**2 / ((2 * Rf * s) ** 2 + float(eps2)) ** 1.5)
+    assert abs(np.linalg.norm(a[0]) - ref) <= 2e-6 * ref      # fp32 position rounding
+    assert a[0, 0] < 0 and abs(a[0, 1]) <= 1e-5 * ref          # radial, inward
+
+
+def test_nbody_shell_theorem():
+    # Newton's shell theorem on a Fibonacci sphere of n equal masses (total M = 1):
+    # outside at distance r the field is M/r^2 toward the centre; inside it vanishes.
+    n = 20000
+    i = np.arange(n) + 0.5
+    phi = np.arccos(1 - 2 * i / n)
+    th = np.pi * (1 + 5**0.5) * i
+    b = np.zeros((n + 2, 4), dtype=np.float32)
+    b[:n, 0] = np.cos(th) * np.sin(phi)
+    b[:n, 1] = np.sin(th) * np.sin(phi)
+    b[:n, 2] = np.cos(phi)
+    b[:n, 3] = 1.0 / n
+    b[n, :3] = [3.0, 0.0, 0.0]
+    b[n + 1, :3] = [0.3, 0.1, 0.0]
+    a = oracle.nbody_accel(b, 1e-6, tgt_begin=n, tgt_count=2)
+    assert abs(a[0, 0] + 1.0 / 9.0) <= 1e-5
+    assert np.linalg.norm(a[1]) <= 1e-5
+
+
+def test_nbody_momentum_conservation_random_cloud():
+    b = inputs.nbody_bodies(1000, seed=11)
+    b[:, 3] = (0.5 + inputs.uniform24(11, 7, 1000)).astype(np.float32)  # unequal masses
+    a, A = oracle.nbody_accel(b, 1e-4, with_mag=True)
+    m = b[:, 3].astype(np.float64)
+    P = (m[:, None] * a).sum(0)
+    assert np.linalg.norm(P) <= 1e-14 * float((m * A).sum())
+    assert np.all(A >= np.linalg.norm(a, axis=1) * (1 - 1e-12))
+
+
+def test_nbody_brute_force_tiny():
+    # Independent brute force in Python (vectorised numpy, different evaluation code).
+    for n in (1, 2, 3, 31, 33):
+        b = inputs.nbody_bodies(n, seed=n)
+        a = oracle.nbody_accel(b, 1e-4)
+        p = b[:, :3].astype(np.float64)
+        m = b[:, 3].astype(np.float64)
+        d = p[None, :, :] - p[:, None, :]
+        r2 = (d**2).sum(-1) + float(np.float32(1e-4))
+        ref = (m[None, :, None] * d / r2[..., None] ** 1.5).sum(1)
+        np.testing.assert_allclose(a, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_nbody_shard_independence():
+    # C-map: out[t] depends only on its own index, so P virtual ranks reproduce the full map.
+    b = inputs.nbody_bodies(96, seed=5)
+    full = oracle.nbody_accel(b, 1e-4)
+    for P in (2, 3, 8):
+        cuts = np.linspace(0, 96, P + 1).astype(int)
+        parts = [oracle.nbody_accel(b, 1e-4, int(lo), int(hi - lo)) for lo, hi in zip(cuts[:-1], cuts[1:])]
+        assert np.array_equal(np.concatenate(parts), full)
+
+
+# oracle_nbody_integrate: forceAccumulator; reading R4
+
+def test_integrator_free_particle_and_constant_acceleration():
+    dt = np.float32(2.0**-10)
+    pos = np.array([[0.25, -0.5, 0.125, 1.0]], dtype=np.float32)
+    vel = np.array([[1.0, 0.0, -2.0, 0.0]], dtype=np.float32)
+    zero = np.zeros((1, 4), dtype=np.float32)
+    p1, v1 = oracle.nbody_integrate(pos, vel, zero, dt)
+    assert np.array_equal(v1, vel.astype(np.float64))
+    np.testing.assert_array_equal(p1[0, :3], pos[0, :3] + vel[0, :3] * float(dt))
+    assert p1[0, 3] == 1.0                                       # mass carried
+    # Semi-implicit Euler under constant a from rest: x_k = x_0 + a dt^2 k(k+1)/2
+    # (explicit Euler would give k(k-1)/2; velocity-Verlet k^2/2).
+    acc = np.array([[1.0, -3.0, 0.5, 0.0]], dtype=np.float32)
+    p, v = pos.copy(), np.zeros((1, 4), dtype=np.float32)
+    for k in range(1, 9):
+        pd, vd = oracle.nbody_integrate(p, v, acc, dt)
+        p, v = pd.astype(np.float32), vd.astype(np.float32)
+        expect = pos[0, :3].astype(np.float64) + acc[0, :3] * float(dt) ** 2 * k * (k + 1) / 2
+        np.testing.assert_array_equal(pd[0, :3], expect)
+
+
+# ====================================================== Black-Scholes
+# oracle_blackscholes: textbook closed form (not in the paper); readings R5-R6
+
+def test_normal_cdf_table():
+    g = _golden("normal_table.json")
+    for x, v in g["table"]:
+        assert round(oracle.normal_cdf(x), g["decimals"]) == pytest.approx(v, abs=1e-12)
+    for x in (0.3, 1.7, 4.2):
+        assert abs(oracle.normal_cdf(-x) - (1 - oracle.normal_cdf(x))) < 1e-15
+
+
+def test_blackscholes_textbook_values():
+    g = _golden("blackscholes_textbook.json")
+    for c in g["cases"]:
+        call, put = oracle.blackscholes(np.array([c["S"]]), np.array([c["X"]]), np.array([c["T"]]),
+                                        c["r"], c["sigma"])
+        assert round(float(call[0]), c["decimals"]) == pytest.approx(c["call"], abs=1e-9)
+        assert round(float(put[0]), c["decimals"]) == pytest.approx(c["put"], abs=1e-9)
+
+
+def test_blackscholes_parity_bounds_monotone():
+    S, X, T = inputs.blackscholes_options(20000, seed=3)
+    r, sg = np.float32(inputs.BS_R), np.float32(inputs.BS_SIGMA)
+    call, put = oracle.blackscholes(S, X, T, r, sg)
+    s, x, t = (a.astype(np.float64) for a in (S, X, T))
+    kx = x * np.exp(-float(r) * t)
+    # put-call parity C - P = S - X e^{-rT}
+    np.testing.assert_allclose(call - put, s - kx, atol=1e-11 * np.maximum(s, x).max(), rtol=0)
+    # no-arbitrage bounds
+    assert np.all(call >= np.maximum(0.0, s - kx) - 1e-12) and np.all(call <= s + 1e-12)
+    assert np.all(put >= np.maximum(0.0, kx - s) - 1e-12) and np.all(put <= kx + 1e-12)
+    # monotone in S: call increasing, put decreasing
+    Ss = np.linspace(5, 30, 200).astype(np.float32)
+    c2, p2 = oracle.blackscholes(Ss, np.full(200, 20, np.float32), np.full(200, 1, np.float32), r, sg)
+    assert np.all(np.diff(c2) > 0) and np.all(np.diff(p2) < 0)
+
+
+def test_blackscholes_zero_volatility_limit():
+    # sigma -> 0: C -> max(0, S - X e^{-rT}), P -> max(0, X e^{-rT} - S) (deterministic forward).
+    S = np.array([10.0, 30.0, 50.0], dtype=np.float32)
+    X = np.array([40.0, 20.0, 50.0], dtype=np.float32)
+    T = np.array([1.0, 2.0, 0.5], dtype=np.float32)
+    r = np.float32(0.05)
+    call, put = oracle.blackscholes(S, X, T, r, np.float32(1e-6))
+    kx = X.astype(np.float64) * np.exp(-float(r) * T)
+    np.testing.assert_allclose(call, np.maximum(0, S - kx), atol=1e-6)
+    np.testing.assert_allclose(put, np.maximum(0, kx - S), atol=1e-6)
+
+
+def test_blackscholes_sums_match_fsum():
+    S, X, T = inputs.blackscholes_options(5000, seed=9)
+    call, put = oracle.blackscholes(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
+    sc, sp = oracle.blackscholes_sums(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
+    assert sc == pytest.approx(math.fsum(call), rel=1e-15)
+    assert sp == pytest.approx(math.fsum(put), rel=1e-15)
+
+
+# ========================================================= Mandelbrot
+# oracle_mandelbrot: exact fp32 emulation (not in the paper); reading R7
+
+def test_mandelbrot_hand_checked_points():
+    g = _golden("mandelbrot_points.json")
+    for cx, cy, n in g["points"]:
+        assert oracle.mandelbrot_point(np.float32(cx), np.float32(cy), g["max_iter"]) == n, (cx, cy)
+
+
+def test_mandelbrot_mirror_symmetry():
+    # cy(8192 - py) = -cy(py) exactly, and y -> -y commutes with every binary32 op.
+    W, dx = 512, 3.0 / 512
+    top = oracle.mandelbrot(W, W, 1, 1, 255, -2.0, -1.5, dx, dx, 256)
+    bot = oracle.mandelbrot(W, W, 511, -1, 255, -2.0, -1.5, dx, dx, 256)
+    assert np.array_equal(top, bot)
+
+
+def test_mandelbrot_cyclic_shards_reassemble():
+    W, dx = 128, 3.0 / 128
+    full = oracle.mandelbrot(W, W, 0, 1, W, -2.0, -1.5, dx, dx, 200)
+    for P in (2, 3, 8):
+        for r in range(P):
+            rows = len(range(r, W, P))
+            shard = oracle.mandelbrot(W, W, r, P, rows, -2.0, -1.5, dx, dx, 200)
+            assert np.array_equal(shard, full[r::P])
+
+
+@pytest.mark.slow
+def test_mandelbrot_frame_checksum():
+    f = _golden("mandelbrot_points.json")["frame"]
+    out = oracle.mandelbrot(f["width"], f["height"], 0, 1, f["height"], f["x0"], f["y0"],
+                            f["dx"], f["dy"], f["max_iter"], threads=os.cpu_count() or 1)
+    assert int(out.sum(dtype=np.int64)) == f["checksum"]
+
+
+# ============================================================= Matmul
+# oracle_matmul_bf16: C = A Bt^T, a map of dot products (not in the paper); reading R8
+
+def _bf16(x):
+    return inputs._f32_to_bf16_bits(np.asarray(x, dtype=np.float32))
+
+
+def test_matmul_identity_and_permutation_exact():
+    K = 16
+    A = inputs.bf16_uniform(5, K, 1, 0)
+    I = _bf16(np.eye(K))
+    np.testing.assert_array_equal(oracle.matmul_bf16(A, I), inputs.bf16_bits_to_f32(A).astype(np.float64))
+    perm = np.random.default_rng(0).permutation(K)
+    Pm = _bf16(np.eye(K)[perm])                      # Bt rows = permuted unit vectors
+    np.testing.assert_array_equal(oracle.matmul_bf16(A, Pm), inputs.bf16_bits_to_f32(A)[:, perm].astype(np.float64))
+
+
+def test_matmul_small_integers_exact_and_not_transposed():
+    rng = np.random.default_rng(1)
+    A = rng.integers(-8, 9, size=(7, 24))
+    Bt = rng.integers(-8, 9, size=(5, 24))
+    ref = A @ Bt.T                                   # exact integer arithmetic
+    out = oracle.matmul_bf16(_bf16(A), _bf16(Bt))
+    np.testing.assert_array_equal(out, ref.astype(np.float64))
+    assert out.shape == (7, 5)
+
+
+def test_matmul_rank1_closed_form():
+    u = np.array([1, -2, 0.5, 4], dtype=np.float32)
+    v = np.array([0.25, 1, -1, 2, 8, -0.5], dtype=np.float32)
+    K = 32
+    A = _bf16(np.outer(u, np.ones(K)))
+    Bt = _bf16(np.outer(v, np.ones(K)))
+    np.testing.assert_array_equal(oracle.matmul_bf16(A, Bt), K * np.outer(u, v).astype(np.float64))
+
+
+def test_matmul_vs_blas_and_entries():
+    A, Bt = inputs.matmul_operands(33, 47, 72, seed=2)
+    ref = inputs.bf16_bits_to_f32(A).astype(np.float64) @ inputs.bf16_bits_to_f32(Bt).astype(np.float64).T
+    C = oracle.matmul_bf16(A, Bt)
+    np.testing.assert_allclose(C, ref, rtol=1e-12, atol=1e-12)
+    rows = np.array([0, 5, 32, 17])
+    cols = np.array([46, 0, 13, 17])
+    Cv, Av = oracle.matmul_bf16_entries(A, Bt, rows, cols)
+    np.testing.assert_array_equal(Cv, C[rows, cols])
+    assert np.all(Av >= np.abs(Cv))
+
+
+# ========================================================= Reductions
+# oracle_reduce_*: PAPER.md L160-163, L188-189; reading R9
+
+def test_reduce_sum_exact_cases():
+    ones = np.ones(1 << 20, dtype=np.float32)
+    assert oracle.reduce("sum", ones, "f32") == float(1 << 20)
+    ints = np.arange(-500, 1500, dtype=np.float32)
+    assert oracle.reduce("sum", ints, "f32") == float(np.arange(-500, 1500).sum())
+    x = inputs.reduce_array(100000, "f32", seed=3)
+    assert oracle.reduce("sum", x, "f32") == pytest.approx(math.fsum(x.astype(np.float64)), rel=1e-15, abs=1e-12)
+    y = inputs.reduce_array(100000, "f64", seed=4)
+    assert oracle.reduce("sum", y, "f64") == pytest.approx(math.fsum(y), rel=1e-14, abs=1e-9)
+
+
+def test_reduce_integer_sums_wrap():
+    x = inputs.reduce_array(10000, "i32", seed=5)
+    assert oracle.reduce("sum", x, "i32") == int(x.astype(np.int64).sum())
+    wrap = np.array([2**31 - 1, 1], dtype=np.int32)
+    assert oracle.reduce("sum", wrap, "i32") == -(2**31)
+    y = inputs.reduce_array(10000, "i64", seed=6)
+    assert oracle.reduce("sum", y, "i64") == sum(int(v) for v in y)
+    wrap64 = np.array([2**63 - 1, 2], dtype=np.int64)
+    assert oracle.reduce("sum", wrap64, "i64") == -(2**63) + 1
+
+
+def test_reduce_min_max_and_nan():
+    for dt in ("f32", "f64", "i32", "i64"):
+        x = inputs.reduce_array(5000, dt, seed=8)
+        assert oracle.reduce("min", x, dt) == min(x.tolist())
+        assert oracle.reduce("max", x, dt) == max(x.tolist())
+    z = np.array([np.nan, 3.0, -1.0, np.nan], dtype=np.float32)
+    assert oracle.reduce("min", z, "f32") == -1.0 and oracle.reduce("max", z, "f32") == 3.0
+    assert math.isnan(oracle.reduce("sum", z, "f32"))
+    assert math.isnan(oracle.reduce("min", np.array([np.nan], np.float32), "f32"))
+
+
+def test_reduce_empty_identity():
+    e = {dt: np.zeros(0, dtype=oracle._RED_DT[dt]) for dt in oracle._RED_DT}
+    assert oracle.reduce("sum", e["f32"], "f32") == 0.0
+    assert oracle.reduce("min", e["f32"], "f32") == math.inf
+    assert oracle.reduce("max", e["f64"], "f64") == -math.inf
+    assert oracle.reduce("min", e["i32"], "i32") == 2**31 - 1
+    assert oracle.reduce("max", e["i64"], "i64") == -(2**63)
