@@ -1,0 +1,450 @@
+#!/usr/bin/env python
+"""bench.py -- the driver's benchmark contract for the Lime map/reduce hot path on B200.
+
+Headline (BASELINE.json metric "map elements/s (N-body interactions/s) and % of FP32/HBM
+roofline, 1-8 B200", config 5): N-Body 2^20 bodies fp32; one STEP = one task-graph pass of the
+paper's N-Body: all-gather of positions (NCCL, N > 1) -> force map
+(lime_map_nbody) -> integrator (lime_map_nbody_integrate). Strong scaling: the 2^20-body
+problem is split by target index over N ranks (torchrun, one process per GPU).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--no-extras]
+
+Rank 0 prints ONE JSON line. At N = 1 the line also carries `configs`: the other
+BASELINE.json configurations measured in the same run (N-Body 4096, Black-Scholes map and
+fused map+reduce, Mandelbrot, matmul, a reduction), each with its own roofline.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import paper_conf_pldi_dubachcrbf12_b200 as lime  # noqa: E402
+from paper_conf_pldi_dubachcrbf12_b200 import dist as ldist  # noqa: E402
+from paper_conf_pldi_dubachcrbf12_b200 import inputs  # noqa: E402
+
+METRIC = "N-body interactions/s (map elements/s)"
+UNIT = "interactions/s"
+EPS2, DT = 1e-4, 1e-3
+FLOP_PER_INTERACTION = 20          # GPU Gems 3 convention
+FP32_LANE_OPS_PER_INTERACTION = 12  # 3 FADD + 3 FFMA (r^2) + 3 FMUL + 3 FFMA (acc)
+SM_MAX_MHZ_NOMINAL = 1965.0
+SMS_B200 = 148
+
+
+# ----------------------------------------------------------------------------- peaks
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained", d["bf16_tflops"]),
+                "sm_max_mhz": d.get("sm_max_mhz", SM_MAX_MHZ_NOMINAL), "source": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0,
+            "sm_max_mhz": SM_MAX_MHZ_NOMINAL, "source": "fallback (B200_PROFILING.md)"}
+
+
+def fp32_peak_tflops(sm_mhz: float) -> float:
+    """FP32 FMA peak derived from unit counts: 148 SMs x 128 FP32 lanes x
+    2 flop x clock. The step-0 microbenchmark measured 124.9-127.9 lane-ops/clk/SM (profiles/)."""
+    return SMS_B200 * 128 * 2 * sm_mhz * 1e6 / 1e12
+
+
+def ncu_traffic(name: str):
+    """dram read+write bytes per launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        return json.load(f).get(name)
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "200", "-i", str(self.gpu)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except (OSError, FileNotFoundError):
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, pw, reasons = [], None, [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+                pw.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        loaded = [s for s in sm if s > 0.5 * (mx or 1)] or sm
+        return {"sm_mhz": float(np.median(loaded)) if loaded else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm), "power_w_max": max(pw) if pw else None}
+
+
+# ----------------------------------------------------------------------------- timing helpers
+def flush_l2(buf):
+    buf.fill_(1)   # write > L2 (2x l2CacheSize) so the next launch starts cold
+
+
+def time_launches(fn, iters, warmup, flush_buf=None):
+    """Median/mean device time of `fn` over `iters` launches, each bracketed by CUDA events on the
+    current stream; the L2 is flushed before every launch (outside the event pair)."""
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
+    for a, b in ev:
+        if flush_buf is not None:
+            flush_l2(flush_buf)
+        a.record()
+        fn()
+        b.record()
+    torch.cuda.synchronize()
+    ms = [a.elapsed_time(b) for a, b in ev]
+    return float(np.median(ms)), float(np.mean(ms))
+
+
+# ----------------------------------------------------------------------------- dist
+def dist_init(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and not dist.is_initialized():
+        if args.impl == "reference":
+            return rank, world, local
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    elif torch.cuda.is_available():
+        torch.cuda.set_device(local)
+    return rank, world, local
+
+
+def barrier(world):
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+def max_over_ranks(x: float, world: int) -> float:
+    if world == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# ----------------------------------------------------------------------------- headline
+def run_nbody(args, rank, world, local):
+    n = args.n
+    bodies = torch.from_numpy(inputs.nbody_bodies(n, seed=5))
+    sim = ldist.NBodySim(bodies, EPS2, DT, f"cuda:{local}")
+    props = torch.cuda.get_device_properties(local)
+    flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    for _ in range(args.warmup):
+        sim.step()
+    barrier(world)
+
+    clocks = ClockSampler(local).start()
+    f_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier(world)
+    t0.record(stream)
+    for k in range(args.steps):
+        flush_l2(flush)
+        sim.gather()
+        f_ev[k][0].record(stream)
+        sim.force_fn(sim.pos_full, sim.begin, sim.count, sim.eps2, sim.accel)
+        f_ev[k][1].record(stream)
+        sim.integrate_fn(sim.pos, sim.vel, sim.accel, sim.dt)
+    t1.record(stream)
+    barrier(world)
+    clk = clocks.stop()
+    ms_local = t0.elapsed_time(t1)
+    force_ms = float(np.mean([a.elapsed_time(b) for a, b in f_ev]))
+    ms_total = max_over_ranks(ms_local, world)
+    force_ms_max = max_over_ranks(force_ms, world)
+
+    interactions_per_step = float(n) * n
+    value = interactions_per_step * args.steps / (ms_total * 1e-3)
+
+    # momentum check (all_reduce of sum m v): |P| / sum m |v| (diagnostic, tiny)
+    mom = sim.momentum()
+    # e2e: host (pinned) state in/out every step through the public API
+    e2e = run_nbody_e2e(args, sim, bodies, world, local)
+
+    peak = fp32_peak_tflops(SM_MAX_MHZ_NOMINAL)
+    per_launch_interactions = float(sim.count) * n
+    achieved = FLOP_PER_INTERACTION * per_launch_interactions / (force_ms * 1e-3) / 1e12
+    obs_mhz = clk.get("sm_mhz") or SM_MAX_MHZ_NOMINAL
+    pipe_frac = (FP32_LANE_OPS_PER_INTERACTION * per_launch_interactions / (force_ms * 1e-3)) / (SMS_B200 * 128 * obs_mhz * 1e6)
+    roofline = {"kernel": "lime::nbody::force_kernel", "bound": "alu", "achieved": achieved, "peak": peak,
+                "unit": "TFLOP/s", "frac": achieved / peak, "traffic": ncu_traffic("nbody_force_1m"),
+                "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 flop x 1965 MHz (microbench: 124.9-127.9 lane-ops/clk/SM)",
+                "flop_per_interaction": FLOP_PER_INTERACTION,
+                "fp32_pipe_frac_at_observed_clock": pipe_frac, "observed_sm_mhz": obs_mhz,
+                "force_ms_per_launch": force_ms, "force_ms_per_launch_max_rank": force_ms_max,
+                "force_share_of_step": force_ms / (ms_local / args.steps)}
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "BASELINE.json configs[4]: N-body all-pairs 2^20 bodies fp32, index-space "
+                                   "sharded, NCCL all-gather per step",
+                       "n_bodies": n, "eps2": EPS2, "dt": DT, "targets_per_gpu": sim.count,
+                       "parallelism": f"target-index shards x{world}" + (" + all_gather" if world > 1 else ""),
+                       "l2": "flushed before every step inside the timed region (2x L2 write); the 16 MiB source "
+                             "array is then re-read from L2 by design (broadcast operand)",
+                       "inputs": "inputs.nbody_bodies(seed=5): U[-1,1)^3, m=1/N, v0=0"},
+            "roofline": roofline, "e2e": e2e, "gpu_launches": 2 * args.steps, "clocks": clk,
+            "momentum_residual": float(mom.norm().item())}
+    return line
+
+
+def run_nbody_e2e(args, sim, bodies, world, local):
+    n = args.n
+    count = sim.count
+    if world == 1:
+        h_pos = bodies.clone().pin_memory()
+        h_vel = torch.zeros((n, 4), dtype=torch.float32).pin_memory()
+        step = lambda: lime.nbody_simulate_host(h_pos, h_vel, 1, EPS2, DT, device=f"cuda:{local}")
+    else:
+        h_pos = sim.pos.cpu().pin_memory()
+        h_vel = sim.vel.cpu().pin_memory()
+        step = lambda: sim.step_host(h_pos, h_vel)
+    for _ in range(max(1, args.warmup)):
+        step()
+    barrier(world)
+    stream = torch.cuda.current_stream()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(args.steps):
+        step()
+    b.record(stream)
+    barrier(world)
+    ms = max_over_ranks(a.elapsed_time(b), world)
+    return {"value": float(n) * n * args.steps / (ms * 1e-3), "unit": UNIT,
+            "h2d_bytes_per_step": 2 * count * 16, "d2h_bytes_per_step": 2 * count * 16,
+            "api": "lime_nbody_simulate_host (C ABI, pinned host buffers)" if world == 1
+            else "dist.NBodySim.step_host (pinned host shards) + C ABI"}
+
+
+# ----------------------------------------------------------------------------- other configs (N = 1)
+def run_extras(peaks, flush):
+    out = {}
+    hbm = peaks["hbm_gbs"]
+    fp32 = fp32_peak_tflops(SM_MAX_MHZ_NOMINAL)
+
+    # config 1: N-Body 4096, one force launch (latency-bound; split-j fills the GPU)
+    b = torch.from_numpy(inputs.nbody_bodies(4096, seed=1)).cuda()
+    acc = torch.empty_like(b)
+    med, mean = time_launches(lambda: lime.map_nbody(b, EPS2, out=acc), 50, 5, flush)
+    inter = 4096.0 * 4096
+    ach = FLOP_PER_INTERACTION * inter / (med * 1e-3) / 1e12
+    out["nbody_4096"] = {"workload": "configs[0]: N-body 4096 bodies fp32, 1 step force map", "value": inter / (med * 1e-3),
+                         "unit": "interactions/s", "ms_per_launch": med,
+                         "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s", "frac": ach / fp32,
+                                      "traffic": ncu_traffic("nbody_force_4096")}}
+    del b, acc
+
+    # config 2: Black-Scholes 2^24 options: map (20 B/option) and fused map+reduce (12 B/option)
+    n = 1 << 24
+    S, X, T = (torch.from_numpy(a).cuda() for a in inputs.blackscholes_options(n, seed=2))
+    call = torch.empty(n, dtype=torch.float32, device="cuda")
+    put = torch.empty_like(call)
+    med, _ = time_launches(lambda: lime.map_blackscholes(S, X, T, inputs.BS_R, inputs.BS_SIGMA, call, put), 30, 5, flush)
+    gbs = 20.0 * n / (med * 1e-3) / 1e9
+    out["blackscholes_map"] = {"workload": "configs[1]: Black-Scholes map, 2^24 options fp32", "value": n / (med * 1e-3),
+                               "unit": "options/s", "ms_per_launch": med,
+                               "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
+                                            "traffic": ncu_traffic("bs_map")}}
+    sums = torch.empty(2, dtype=torch.float64, device="cuda")
+    med, _ = time_launches(lambda: lime.map_reduce_blackscholes_sum(S, X, T, inputs.BS_R, inputs.BS_SIGMA, sums), 30, 5, flush)
+    gbs = 12.0 * n / (med * 1e-3) / 1e9
+    out["blackscholes_map_reduce"] = {"workload": "configs[1]: Black-Scholes fused map+reduce of total premium, 2^24 options",
+                                      "value": n / (med * 1e-3), "unit": "options/s", "ms_per_launch": med,
+                                      "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s",
+                                                   "frac": gbs / hbm, "traffic": ncu_traffic("bs_map_reduce")}}
+    del S, X, T, call, put
+
+    # config 3: Mandelbrot 8192^2, max 1024 (11,856,987,162 iterations; 8 FP32 lane-ops each)
+    W = 8192
+    d = 3.0 / W
+    cnt = torch.empty((W, W), dtype=torch.int32, device="cuda")
+    med, _ = time_launches(lambda: lime.map_mandelbrot(W, W, -2.0, -1.5, d, d, 1024, out=cnt), 10, 2, flush)
+    iters = float(cnt.sum(dtype=torch.int64).item())
+    lane_ops = 8.0 * iters / (med * 1e-3)
+    peak_lane = SMS_B200 * 128 * SM_MAX_MHZ_NOMINAL * 1e6
+    out["mandelbrot"] = {"workload": "configs[2]: Mandelbrot 8192x8192, max_iter 1024, int32 bit-exact",
+                         "value": W * W / (med * 1e-3), "unit": "pixels/s", "iterations_per_s": iters / (med * 1e-3),
+                         "ms_per_launch": med, "checksum": int(iters),
+                         "roofline": {"bound": "alu", "achieved": lane_ops / 1e12, "peak": peak_lane / 1e12,
+                                      "unit": "T FP32 lane-ops/s", "frac": lane_ops / peak_lane,
+                                      "traffic": ncu_traffic("mandelbrot")}}
+    del cnt
+
+    # config 4: matmul 8192^3 bf16 -> fp32 (tcgen05)
+    M = N = K = 8192
+    try:
+        A = torch.from_numpy(inputs.bf16_uniform(M, K, 4, 0).view(np.int16)).cuda().view(torch.bfloat16)
+        Bt = torch.from_numpy(inputs.bf16_uniform(N, K, 4, 1).view(np.int16)).cuda().view(torch.bfloat16)
+        Cm = torch.empty((M, N), dtype=torch.float32, device="cuda")
+        med, _ = time_launches(lambda: lime.map_matmul_bf16(A, Bt, Cm), 20, 3, flush)
+        tf = 2.0 * M * N * K / (med * 1e-3) / 1e12
+        cub, _ = time_launches(lambda: torch.matmul(A, Bt.t()), 20, 3, flush)
+        out["matmul"] = {"workload": "configs[3]: matmul 8192^3 bf16 in, fp32 accumulate/out (tcgen05)",
+                         "value": M * N / (med * 1e-3), "unit": "dot products/s", "ms_per_launch": med,
+                         "tflops": tf, "cublas_bf16_out_ms": cub,
+                         "roofline": {"bound": "tensor", "achieved": tf, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
+                                      "frac": tf / peaks["bf16_tflops"], "traffic": ncu_traffic("matmul")}}
+        del A, Bt, Cm
+    except lime.LimeError as e:
+        out["matmul"] = {"workload": "configs[3]", "unavailable": str(e)}
+
+    # reduction `!`: sum over 2^28 fp32 (1 GiB)
+    x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
+    r = torch.empty((), dtype=torch.float32, device="cuda")
+    med, _ = time_launches(lambda: lime.reduce_sum(x, r), 20, 3, flush)
+    gbs = 4.0 * (1 << 28) / (med * 1e-3) / 1e9
+    out["reduce_sum_f32"] = {"workload": "reduce ! sum over 2^28 fp32", "value": (1 << 28) / (med * 1e-3),
+                             "unit": "elements/s", "ms_per_launch": med,
+                             "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
+                                          "traffic": ncu_traffic("reduce_sum_f32")}}
+    del x
+    return out
+
+
+# ----------------------------------------------------------------------------- CPU oracle
+def cpu_oracle_sample(n: int, targets: int):
+    """The oracle as it stands (single-threaded C, fp64): accelerations of `targets` targets
+    against all n sources of the same workload. Returns (interactions/s, seconds)."""
+    import oracle
+    b = inputs.nbody_bodies(n, seed=5)
+    oracle.lib()
+    t = time.perf_counter()
+    oracle.nbody_accel(b, np.float32(EPS2), 0, targets)
+    dt = time.perf_counter() - t
+    return targets * float(n) / dt, dt
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return None
+    import oracle
+    n = args.n
+    b = inputs.nbody_bodies(n, seed=5)
+    vel = np.zeros((args.ref_targets, 4), dtype=np.float32)
+    oracle.lib()
+    times = []
+    for k in range(args.warmup + args.steps):
+        t = time.perf_counter()
+        lo = (k * args.ref_targets) % n
+        acc = oracle.nbody_accel(b, np.float32(EPS2), lo, args.ref_targets)
+        a4 = np.zeros((args.ref_targets, 4), dtype=np.float32)
+        a4[:, :3] = acc
+        oracle.nbody_integrate(b[lo:lo + args.ref_targets], vel, a4, np.float32(DT))
+        if k >= args.warmup:
+            times.append(time.perf_counter() - t)
+    per_step = float(np.mean(times))
+    value = args.ref_targets * float(n) / per_step
+    sample = f"{args.ref_targets} targets x {n} sources (+ integrator) of the config-5 workload per step"
+    return {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": per_step * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": "BASELINE.json configs[4]: N-body 2^20 bodies (oracle sample)", "n_bodies": n},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+# ----------------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["lime", "reference"], default="lime")
+    ap.add_argument("--n", type=int, default=1 << 20)
+    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--cpu-targets", type=int, default=3072)
+    ap.add_argument("--ref-targets", type=int, default=512)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3) if args.impl == "lime" else args.warmup
+
+    rank, world, local = dist_init(args)
+    if args.impl == "reference":
+        line = run_reference(args, rank, world)
+        if line is not None:
+            print(json.dumps(line), flush=True)
+        return
+
+    lime.load()
+    peaks = measured_peaks()
+    line = run_nbody(args, rank, world, local)
+    if rank == 0 and world == 1:
+        if not args.no_extras:
+            props = torch.cuda.get_device_properties(local)
+            flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
+            line["configs"] = run_extras(peaks, flush)
+        v, secs = cpu_oracle_sample(args.n, args.cpu_targets)
+        line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": f"{args.cpu_targets} targets x {args.n} sources of step 0 "
+                                          f"({secs:.1f} s, single-threaded C fp64)"}
+    elif rank == 0:
+        line["cpu_baseline"] = None
+    line["peaks"] = peaks
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

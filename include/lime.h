@@ -1,0 +1,213 @@
+/*
+ * lime.h -- C ABI of liblime.so, the B200-native (sm_100a) map `@` / reduce `!`
+ * hot path of Lime (Dubach, Cheng, Rabbah, Bacon, Fink, PLDI 2012).
+ *
+ * Citations Lnnn are lines of the decoded `fulltext` of PAPER.md.
+ *
+ * ---------------------------------------------------------------------------
+ * Conventions (apply to every entry point unless its comment says otherwise)
+ * ---------------------------------------------------------------------------
+ * Semantics. A map `@` applies a pure element function to each element of an
+ *   immutable value array and returns a NEW array (L149-157 §3.2; purity from
+ *   "static and local" + value-typed arguments, L184-189). A reduce `!`
+ *   combines elements with a binary combinator of one type (L160-163). Every
+ *   map here computes out[t] = f(in[begin + t], broadcast operands) for
+ *   t in [0, count); the result does not depend on how many threads run it
+ *   (L205-208).
+ * Pointers. Unless the name ends in `_host`, every array pointer is a DEVICE
+ *   pointer (e.g. a torch CUDA tensor's data_ptr()) owned by the caller. The
+ *   library keeps no pointer after returning and allocates/frees nothing.
+ * Layout. Dense row-major arrays of primitives (L297-301). float4 operands and
+ *   `*_workspace` buffers must be 16-byte aligned.
+ * Value semantics. Inputs are never written (L136-143); an output range that
+ *   overlaps an input range is rejected with LIME_ERR_ALIASING. The integrator
+ *   is the documented exception (in/out state; it is the paper's stateful sink
+ *   task, L112-113, not a filter).
+ * Streams. `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *   stream). All work is enqueued asynchronously on it; the library never
+ *   synchronises, except `_host` entry points, which synchronise `stream`
+ *   before returning (their outputs are host memory).
+ * Workspaces. Entry points taking (ws, ws_bytes) need a device scratch buffer
+ *   of at least the size returned by the matching *_workspace_bytes() query,
+ *   ZERO-FILLED before its first use; every call leaves it zero-filled again
+ *   (self-resetting counters), so one buffer can be reused by consecutive
+ *   calls on the same stream. Two calls that run concurrently need two
+ *   workspaces.
+ * Errors. Every entry point returns lime_status; no C++ exception crosses the
+ *   ABI. Validation order: arguments (LIME_ERR_INVALID_ARG) -> alignment
+ *   (LIME_ERR_MISALIGNED) -> aliasing (LIME_ERR_ALIASING) -> device check
+ *   (LIME_ERR_UNSUPPORTED: current device is not compute capability 10.0)
+ *   -> workspace size (LIME_ERR_WORKSPACE) -> launch (LIME_ERR_CUDA from
+ *   cudaGetLastError). Nothing is enqueued when a non-OK status is returned.
+ *   Faults inside asynchronous work surface at the next synchronisation, as
+ *   in CUDA. lime_last_error() gives a thread-local message for the last
+ *   non-OK status. Count 0 is a valid no-op for maps.
+ */
+#ifndef LIME_H
+#define LIME_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    LIME_OK = 0,
+    LIME_ERR_INVALID_ARG = 1,
+    LIME_ERR_MISALIGNED = 2,
+    LIME_ERR_ALIASING = 3,
+    LIME_ERR_UNSUPPORTED = 4,
+    LIME_ERR_CUDA = 5,
+    LIME_ERR_WORKSPACE = 6
+} lime_status;
+
+#define LIME_ABI_VERSION 1
+
+/* ABI version (LIME_ABI_VERSION). */
+int lime_abi_version(void);
+/* Static string naming a status code. */
+const char *lime_status_str(int status);
+/* Thread-local detail for the last non-OK status returned on this thread ("" if none). */
+const char *lime_last_error(void);
+/* LIME_OK iff the current CUDA device is an sm_100 part (B200); else LIME_ERR_UNSUPPORTED. */
+lime_status lime_device_check(void);
+/* Number of SMs of the current device (0 if no device). */
+int lime_num_sms(void);
+/* Test/tuning hook (paper L204-205 "number of threads ... requested by the user", L380-385
+ * offline tuning): override the launch configuration of the next calls on this thread.
+ * grid_ctas = 0 / block_threads = 0 / per_thread = 0 restore the automatic choice. Each
+ * kernel documents which knobs it honours; results of maps never depend on them. */
+void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
+
+/* ===========================================================================
+ * N-Body all-pairs force map (the paper's workload: L106-114 task graph,
+ * L108-112 float[[][4]] particles -> per-particle force, L156-158 "each
+ * application of the map function computes the force interactions between a
+ * particle p and all other particles", L173-174 "n^2 force calculation").
+ * Formula (paper omits it, L157-158; R1-R3):
+ *   accel[t] = sum_{j=0}^{n_src-1} m_j (p_j - p_i) (|p_j - p_i|^2 + eps2)^{-3/2},
+ *   i = tgt_begin + t, G = 1, self term included (exactly 0).
+ *   bodies  [n_src][4] float (x, y, z, m), 16-B aligned  -- the mapped array AND
+ *           the broadcast operand staged through shared memory (L234-255).
+ *   accel   [tgt_count][4] float (ax, ay, az, 0), 16-B aligned, must not
+ *           overlap bodies.
+ *   eps2    Plummer softening, finite and > 0 (eps2 <= 0 makes the self term 0/0).
+ *   0 <= tgt_begin, 0 <= tgt_count, tgt_begin + tgt_count <= n_src.
+ * Summation order (deterministic, independent of launch config and of the
+ * target shard): sources are cut into 256-body chunks; each chunk is summed in
+ * j order into a chunk partial; chunk partials are added in order into one of
+ * S = nbody_splits(n_src) split partials; split partials are added in s order.
+ * Launch override: grid ignored; block_threads in {128, 256}; per_thread in {1, 2, 4, 8}.
+ * =========================================================================== */
+size_t lime_map_nbody_workspace_bytes(int64_t n_src, int64_t tgt_count);
+int lime_nbody_splits(int64_t n_src);
+lime_status lime_map_nbody(const float *bodies, int64_t n_src, int64_t tgt_begin,
+                           int64_t tgt_count, float eps2, float *accel,
+                           void *ws, size_t ws_bytes, void *stream);
+
+/* N-Body integrator (the `forceAccumulator` sink, L112-114; R4):
+ * semi-implicit Euler on n bodies, in place:
+ *   vel.xyz += accel.xyz * dt ;  pos.xyz += vel.xyz * dt ;  pos.w (mass), vel.w kept.
+ * pos, vel, accel: [n][4] float, 16-B aligned; accel must not overlap pos/vel;
+ * pos and vel must not overlap each other. dt finite.
+ * Launch override: grid_ctas honoured. */
+lime_status lime_map_nbody_integrate(float *pos, float *vel, const float *accel, int64_t n,
+                                     float dt, void *stream);
+
+/* One complete N-Body simulation step through HOST buffers (end-to-end entry,
+ * PAPER.md Fig. 6 / §4.3 L275-286 host<->device transport): copies h_pos and
+ * h_vel ([n][4] float, host memory, pinned for best speed) to the device
+ * scratch `ws`, runs `steps` x (lime_map_nbody over all n targets +
+ * lime_map_nbody_integrate), copies the new state back into h_pos / h_vel and
+ * synchronises `stream`. ws: lime_nbody_simulate_host_workspace_bytes(n) bytes,
+ * device, zero-filled before first use. */
+size_t lime_nbody_simulate_host_workspace_bytes(int64_t n);
+lime_status lime_nbody_simulate_host(float *h_pos, float *h_vel, int64_t n, int32_t steps,
+                                     float eps2, float dt, void *ws, size_t ws_bytes,
+                                     void *stream);
+
+/* ===========================================================================
+ * Black-Scholes European options (BASELINE.json config 2; not in the paper --
+ * a transcendental streaming map of the kind it evaluates, SURVEY.md §0.2;
+ * DESIGN.md R5). Per option i:
+ *   d1 = (ln(S/X) + (r + sigma^2/2) T) / (sigma sqrt T), d2 = d1 - sigma sqrt T
+ *   call[i] = S N(d1) - X e^{-rT} N(d2),  put[i] = X e^{-rT} N(-d2) - S N(-d1)
+ * S, X, T: [n] float (SoA), 16-B aligned; call, put: [n] float, 16-B aligned,
+ * no overlap with inputs or each other. S, X, T > 0, sigma > 0 (not checked
+ * per element: a non-positive element yields NaN/inf in its own outputs only).
+ * N() uses the Abramowitz-Stegun 26.2.17 approximation (|err| < 7.5e-8).
+ * Launch override: grid_ctas, block_threads honoured.
+ * =========================================================================== */
+lime_status lime_map_blackscholes(const float *S, const float *X, const float *T, int64_t n,
+                                  float r, float sigma, float *call, float *put, void *stream);
+
+/* Fused map+reduce (`!` over `@` without materialising the map, L160-163,
+ * L188-189; R6): sums[0] = sum_i call[i], sums[1] = sum_i put[i]
+ * (device double[2]), accumulated in fp64 from the CTA level up, CTA partials
+ * combined in fixed index order by the last CTA (deterministic for a given
+ * launch configuration). ws: lime_reduce_workspace_bytes() bytes. */
+lime_status lime_map_reduce_blackscholes_sum(const float *S, const float *X, const float *T,
+                                             int64_t n, float r, float sigma, double *sums,
+                                             void *ws, size_t ws_bytes, void *stream);
+
+/* ===========================================================================
+ * Mandelbrot escape counts (BASELINE.json config 3; not in the paper; an
+ * integer-output compute-bound map; R7). Bit-exact binary32:
+ *   cx = x0 + px*dx, cy = y0 + py*dy, z0 = 0; count n while n < max_iter and
+ *   x^2 + y^2 <= 4: x <- (x^2 - y^2) + cx, y <- (xy + xy) + cy.
+ * Output counts [row_count][width] int32; output row k is image row
+ * py = row_first + k*row_stride (row_stride = P, row_first = rank gives the
+ * cyclic multi-GPU shard). width, height > 0; 0 <= row_first < height;
+ * row_stride >= 1; every addressed py < height; max_iter >= 0.
+ * ws: lime_mandelbrot_workspace_bytes() bytes (tile-queue counters).
+ * Launch override: grid_ctas honoured.
+ * =========================================================================== */
+size_t lime_mandelbrot_workspace_bytes(void);
+lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first,
+                                int32_t row_stride, int32_t row_count, float x0, float y0,
+                                float dx, float dy, int32_t max_iter, int32_t *counts,
+                                void *ws, size_t ws_bytes, void *stream);
+
+/* ===========================================================================
+ * Dense matrix multiply as a map of dot products (BASELINE.json config 4; not
+ * in the paper; R8): C[i][j] = sum_k A[i][k] * Bt[j][k].
+ * A [M][K] bf16 bits (uint16), Bt [N][K] bf16 bits (K-major both), C [M][N]
+ * float (fp32 accumulate, tcgen05 tensor cores). M, N >= 1; K >= 8 and
+ * K % 8 == 0 (16-byte TMA row stride); A, Bt, C 16-B aligned; C must not
+ * overlap A or Bt.
+ * =========================================================================== */
+lime_status lime_map_matmul_bf16(const uint16_t *A, const uint16_t *Bt, float *C, int64_t M,
+                                 int64_t N, int64_t K, void *stream);
+
+/* ===========================================================================
+ * Reductions `!` over an array x[n] (L160-163; L188-189 "the compiler may
+ * infer a parallel reduction"; R9). Tree: per-thread fold ->
+ * warp shuffle -> CTA -> last CTA combines the CTA partials in index order.
+ * `out` is a DEVICE pointer to one element of the result type:
+ *   sum_f32 -> float (accumulated in fp64 above the thread level)
+ *   sum_f64 -> double, sum_i32 -> int32 (wraps), sum_i64 -> int64 (wraps)
+ *   min/max -> the element type; NaN ignored (fmin/fmax); NaN only if all NaN.
+ * Empty input writes the identity (0, +inf/-inf, INT_MAX/INT_MIN).
+ * x needs only natural alignment of its element type. ws:
+ * lime_reduce_workspace_bytes() bytes. Launch override: grid_ctas, block_threads.
+ * =========================================================================== */
+size_t lime_reduce_workspace_bytes(void);
+lime_status lime_reduce_sum_f32(const float *x, int64_t n, float *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_sum_f64(const double *x, int64_t n, double *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_sum_i32(const int32_t *x, int64_t n, int32_t *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_sum_i64(const int64_t *x, int64_t n, int64_t *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_min_f32(const float *x, int64_t n, float *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_min_f64(const double *x, int64_t n, double *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_min_i32(const int32_t *x, int64_t n, int32_t *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_min_i64(const int64_t *x, int64_t n, int64_t *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_max_f32(const float *x, int64_t n, float *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_max_f64(const double *x, int64_t n, double *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_max_i32(const int32_t *x, int64_t n, int32_t *out, void *ws, size_t ws_bytes, void *stream);
+lime_status lime_reduce_max_i64(const int64_t *x, int64_t n, int64_t *out, void *ws, size_t ws_bytes, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIME_H */

@@ -1,0 +1,264 @@
+"""paper_conf_pldi_dubachcrbf12_b200 -- B200-native map `@` / reduce `!` hot path of Lime
+(Dubach et al., PLDI 2012).
+
+Thin Python binding over the C ABI of liblime.so (contract: include/lime.h). This module only
+marshals arguments: torch CUDA tensors -> device pointers, the current CUDA stream, zeroed
+workspaces. Every step of the path runs in the CUDA kernels; there is no CPU fallback -- if the
+library is missing, load() raises.
+
+Public API (names follow the ABI):
+    map_nbody, map_nbody_integrate, nbody_simulate_host,
+    map_blackscholes, map_reduce_blackscholes_sum,
+    map_mandelbrot, map_matmul_bf16,
+    reduce_sum / reduce_min / reduce_max (f32, f64, i32, i64),
+    launch_override (context manager; PAPER.md L204-205 user-chosen thread counts).
+"""
+from __future__ import annotations
+
+import contextlib
+import ctypes as C
+import os
+import threading
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblime.so")
+
+STATUS = {0: "LIME_OK", 1: "LIME_ERR_INVALID_ARG", 2: "LIME_ERR_MISALIGNED", 3: "LIME_ERR_ALIASING",
+          4: "LIME_ERR_UNSUPPORTED", 5: "LIME_ERR_CUDA", 6: "LIME_ERR_WORKSPACE"}
+
+
+class LimeError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+        self.status = status
+
+
+_lib = None
+_lock = threading.Lock()
+_p, _i64, _i32, _f, _sz, _int = C.c_void_p, C.c_int64, C.c_int32, C.c_float, C.c_size_t, C.c_int
+
+# Signatures of every symbol include/lime.h declares (tests check the two agree).
+SIGNATURES = {
+    "lime_abi_version": (_int, []),
+    "lime_status_str": (C.c_char_p, [_int]),
+    "lime_last_error": (C.c_char_p, []),
+    "lime_device_check": (_int, []),
+    "lime_num_sms": (_int, []),
+    "lime_set_launch_override": (None, [_int, _int, _int]),
+    "lime_map_nbody_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_nbody_splits": (_int, [_i64]),
+    "lime_map_nbody": (_int, [_p, _i64, _i64, _i64, _f, _p, _p, _sz, _p]),
+    "lime_map_nbody_integrate": (_int, [_p, _p, _p, _i64, _f, _p]),
+    "lime_nbody_simulate_host_workspace_bytes": (_sz, [_i64]),
+    "lime_nbody_simulate_host": (_int, [_p, _p, _i64, _i32, _f, _f, _p, _sz, _p]),
+    "lime_map_blackscholes": (_int, [_p, _p, _p, _i64, _f, _f, _p, _p, _p]),
+    "lime_map_reduce_blackscholes_sum": (_int, [_p, _p, _p, _i64, _f, _f, _p, _p, _sz, _p]),
+    "lime_mandelbrot_workspace_bytes": (_sz, []),
+    "lime_map_mandelbrot": (_int, [_i32, _i32, _i32, _i32, _i32, _f, _f, _f, _f, _i32, _p, _p, _sz, _p]),
+    "lime_map_matmul_bf16": (_int, [_p, _p, _p, _i64, _i64, _i64, _p]),
+    "lime_reduce_workspace_bytes": (_sz, []),
+}
+for _op in ("sum", "min", "max"):
+    for _dt in ("f32", "f64", "i32", "i64"):
+        SIGNATURES[f"lime_reduce_{_op}_{_dt}"] = (_int, [_p, _i64, _p, _p, _sz, _p])
+
+
+def load(path: str | None = None):
+    """Load liblime.so (raises if it is missing -- never falls back)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            p = path or LIB_PATH
+            if not os.path.exists(p):
+                raise RuntimeError(f"liblime.so not built ({p}); run `python -m paper_conf_pldi_dubachcrbf12_b200.build`")
+            lib = C.CDLL(p)
+            for name, (res, args) in SIGNATURES.items():
+                fn = getattr(lib, name)
+                fn.restype = res
+                fn.argtypes = args
+            _lib = lib
+    return _lib
+
+
+def _check(status: int, what: str):
+    if status != 0:
+        raise LimeError(status, f"{what}: {load().lime_last_error().decode()}")
+
+
+def _stream(device) -> int:
+    return torch.cuda.current_stream(device).cuda_stream
+
+
+def _dev_tensor(t: torch.Tensor, dtype, name: str, ndim_last: int | None = None):
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if ndim_last is not None and (t.dim() != 2 or t.shape[1] != ndim_last):
+        raise ValueError(f"{name} must have shape [n][{ndim_last}]")
+    return t
+
+
+# Zero-filled, self-resetting workspaces, one per (device, stream, kind).
+_ws_cache: dict = {}
+
+
+def workspace(device, kind: str, nbytes: int) -> torch.Tensor:
+    dev = torch.device(device)
+    key = (dev.index, _stream(dev), kind)
+    buf = _ws_cache.get(key)
+    if buf is None or buf.numel() < nbytes:
+        buf = torch.zeros(max(int(nbytes), 256), dtype=torch.uint8, device=dev)
+        _ws_cache[key] = buf
+    return buf
+
+
+@contextlib.contextmanager
+def launch_override(grid_ctas: int = 0, block_threads: int = 0, per_thread: int = 0):
+    """Override the launch configuration on this thread (results never depend on it)."""
+    L = load()
+    L.lime_set_launch_override(grid_ctas, block_threads, per_thread)
+    try:
+        yield
+    finally:
+        L.lime_set_launch_override(0, 0, 0)
+
+
+def num_sms() -> int:
+    return int(load().lime_num_sms())
+
+
+# ------------------------------------------------------------------------ N-Body
+def nbody_splits(n_src: int) -> int:
+    return int(load().lime_nbody_splits(n_src))
+
+
+def map_nbody(bodies: torch.Tensor, eps2: float, tgt_begin: int = 0, tgt_count: int | None = None,
+              out: torch.Tensor | None = None) -> torch.Tensor:
+    """accel[t] for targets [tgt_begin, tgt_begin+tgt_count) of bodies [n][4] (x,y,z,m)."""
+    L = load()
+    _dev_tensor(bodies, torch.float32, "bodies", 4)
+    n = bodies.shape[0]
+    if tgt_count is None:
+        tgt_count = n - tgt_begin
+    if out is None:
+        out = torch.empty((max(tgt_count, 0), 4), dtype=torch.float32, device=bodies.device)
+    _dev_tensor(out, torch.float32, "out", 4)
+    nbytes = L.lime_map_nbody_workspace_bytes(n, max(tgt_count, 0))
+    ws = workspace(bodies.device, "nbody", nbytes)
+    _check(L.lime_map_nbody(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
+                            ws.data_ptr(), ws.numel(), _stream(bodies.device)), "lime_map_nbody")
+    return out
+
+
+def map_nbody_integrate(pos: torch.Tensor, vel: torch.Tensor, accel: torch.Tensor, dt: float) -> None:
+    """In-place semi-implicit Euler step of pos/vel ([n][4] each)."""
+    L = load()
+    for t, nm in ((pos, "pos"), (vel, "vel"), (accel, "accel")):
+        _dev_tensor(t, torch.float32, nm, 4)
+    _check(L.lime_map_nbody_integrate(pos.data_ptr(), vel.data_ptr(), accel.data_ptr(), pos.shape[0], dt,
+                                      _stream(pos.device)), "lime_map_nbody_integrate")
+
+
+def nbody_simulate_host(h_pos: torch.Tensor, h_vel: torch.Tensor, steps: int, eps2: float, dt: float,
+                        device="cuda") -> None:
+    """End-to-end: host (pinned) state in, `steps` force+integrate steps on the GPU, host state out."""
+    L = load()
+    for t, nm in ((h_pos, "h_pos"), (h_vel, "h_vel")):
+        if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.dim() != 2 or t.shape[1] != 4:
+            raise ValueError(f"{nm} must be a contiguous host float32 [n][4] tensor")
+    n = h_pos.shape[0]
+    dev = torch.device(device)
+    ws = workspace(dev, "nbody_host", L.lime_nbody_simulate_host_workspace_bytes(n))
+    _check(L.lime_nbody_simulate_host(h_pos.data_ptr(), h_vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(),
+                                      ws.numel(), _stream(dev)), "lime_nbody_simulate_host")
+
+
+# ------------------------------------------------------------------ Black-Scholes
+def map_blackscholes(S, X, T, r: float, sigma: float, call=None, put=None):
+    L = load()
+    for t, nm in ((S, "S"), (X, "X"), (T, "T")):
+        _dev_tensor(t, torch.float32, nm)
+    n = S.numel()
+    call = torch.empty(n, dtype=torch.float32, device=S.device) if call is None else call
+    put = torch.empty(n, dtype=torch.float32, device=S.device) if put is None else put
+    _check(L.lime_map_blackscholes(S.data_ptr(), X.data_ptr(), T.data_ptr(), n, r, sigma, call.data_ptr(),
+                                   put.data_ptr(), _stream(S.device)), "lime_map_blackscholes")
+    return call, put
+
+
+def map_reduce_blackscholes_sum(S, X, T, r: float, sigma: float, out=None) -> torch.Tensor:
+    """Device float64[2] = (sum call, sum put), fused (the map is never materialised)."""
+    L = load()
+    for t, nm in ((S, "S"), (X, "X"), (T, "T")):
+        _dev_tensor(t, torch.float32, nm)
+    out = torch.empty(2, dtype=torch.float64, device=S.device) if out is None else out
+    ws = workspace(S.device, "reduce", L.lime_reduce_workspace_bytes())
+    _check(L.lime_map_reduce_blackscholes_sum(S.data_ptr(), X.data_ptr(), T.data_ptr(), S.numel(), r, sigma,
+                                              out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(S.device)),
+           "lime_map_reduce_blackscholes_sum")
+    return out
+
+
+# ----------------------------------------------------------------- Mandelbrot
+def map_mandelbrot(width: int, height: int, x0: float, y0: float, dx: float, dy: float, max_iter: int,
+                   row_first: int = 0, row_stride: int = 1, row_count: int | None = None,
+                   device="cuda", out=None) -> torch.Tensor:
+    L = load()
+    if row_count is None:
+        row_count = len(range(row_first, height, row_stride))
+    dev = torch.device(device)
+    out = torch.empty((row_count, width), dtype=torch.int32, device=dev) if out is None else out
+    ws = workspace(dev, "mandel", L.lime_mandelbrot_workspace_bytes())
+    _check(L.lime_map_mandelbrot(width, height, row_first, row_stride, row_count, x0, y0, dx, dy, max_iter,
+                                 out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_mandelbrot")
+    return out
+
+
+# --------------------------------------------------------------------- Matmul
+def map_matmul_bf16(A: torch.Tensor, Bt: torch.Tensor, out=None) -> torch.Tensor:
+    """C[M][N] fp32 = A[M][K] . Bt[N][K]^T (bf16 in, tcgen05 tensor cores)."""
+    L = load()
+    _dev_tensor(A, torch.bfloat16, "A")
+    _dev_tensor(Bt, torch.bfloat16, "Bt")
+    M, K = A.shape
+    N = Bt.shape[0]
+    if Bt.shape[1] != K:
+        raise ValueError("A and Bt must share K")
+    out = torch.empty((M, N), dtype=torch.float32, device=A.device) if out is None else out
+    _check(L.lime_map_matmul_bf16(A.data_ptr(), Bt.data_ptr(), out.data_ptr(), M, N, K, _stream(A.device)),
+           "lime_map_matmul_bf16")
+    return out
+
+
+# ----------------------------------------------------------------- Reductions
+_RED_DT = {torch.float32: "f32", torch.float64: "f64", torch.int32: "i32", torch.int64: "i64"}
+
+
+def _reduce(op: str, x: torch.Tensor, out=None) -> torch.Tensor:
+    L = load()
+    if x.dtype not in _RED_DT:
+        raise TypeError(f"unsupported dtype {x.dtype}")
+    _dev_tensor(x, x.dtype, "x")
+    out = torch.empty((), dtype=x.dtype, device=x.device) if out is None else out
+    ws = workspace(x.device, "reduce", L.lime_reduce_workspace_bytes())
+    fn = getattr(L, f"lime_reduce_{op}_{_RED_DT[x.dtype]}")
+    _check(fn(x.data_ptr(), x.numel(), out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(x.device)),
+           f"lime_reduce_{op}")
+    return out
+
+
+def reduce_sum(x, out=None):
+    return _reduce("sum", x, out)
+
+
+def reduce_min(x, out=None):
+    return _reduce("min", x, out)
+
+
+def reduce_max(x, out=None):
+    return _reduce("max", x, out)

@@ -1,0 +1,342 @@
+// abi.cu -- the extern "C" boundary of liblime.so (contract: include/lime.h).
+//
+// Host-side only: argument validation (in the documented order), device check, workspace
+// check, then the launcher in the kernel translation unit. Validation never touches the
+// GPU, so the error paths are testable on a machine without one.
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+
+#include "../../include/lime.h"
+#include "common.cuh"
+#include "kernels.h"
+
+namespace lime {
+
+static thread_local char g_last_error[512] = "";
+static thread_local LaunchOverride g_override;
+
+const LaunchOverride& launch_override() { return g_override; }
+
+int device_num_sms() {
+    static int cached[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return kNumSMsB200;
+    if (cached[dev] == 0) {
+        int sms = 0;
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) {
+            cudaGetLastError();
+            return kNumSMsB200;
+        }
+        cached[dev] = sms;
+    }
+    return cached[dev];
+}
+
+static lime_status fail(lime_status s, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_last_error, sizeof g_last_error, fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+static bool overlap(const void* a, size_t abytes, const void* b, size_t bbytes) {
+    if (abytes == 0 || bbytes == 0) return false;
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(a), b0 = reinterpret_cast<uintptr_t>(b);
+    return a0 < b0 + bbytes && b0 < a0 + abytes;
+}
+
+static lime_status check_device() {
+    static int ok_cache[64] = {0};   // 0 unknown, 1 ok, 2 bad
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(LIME_ERR_UNSUPPORTED, "no CUDA device: %s", cudaGetErrorString(e));
+    }
+    if (dev >= 0 && dev < 64 && ok_cache[dev] == 1) return LIME_OK;
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    if (major != 10 || minor != 0) {
+        if (dev >= 0 && dev < 64) ok_cache[dev] = 2;
+        return fail(LIME_ERR_UNSUPPORTED, "device %d is sm_%d%d; liblime is built for sm_100a (B200) only",
+                    dev, major, minor);
+    }
+    if (dev >= 0 && dev < 64) ok_cache[dev] = 1;
+    return LIME_OK;
+}
+
+static lime_status launched(cudaError_t e, const char* what) {
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(LIME_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+    }
+    return LIME_OK;
+}
+
+}  // namespace lime
+
+using namespace lime;
+
+#define LIME_TRY(expr)                              \
+    do {                                            \
+        const lime_status s__ = (expr);             \
+        if (s__ != LIME_OK) return s__;             \
+    } while (0)
+
+extern "C" {
+
+int lime_abi_version(void) { return LIME_ABI_VERSION; }
+
+const char* lime_status_str(int s) {
+    switch (s) {
+        case LIME_OK: return "LIME_OK";
+        case LIME_ERR_INVALID_ARG: return "LIME_ERR_INVALID_ARG";
+        case LIME_ERR_MISALIGNED: return "LIME_ERR_MISALIGNED";
+        case LIME_ERR_ALIASING: return "LIME_ERR_ALIASING";
+        case LIME_ERR_UNSUPPORTED: return "LIME_ERR_UNSUPPORTED";
+        case LIME_ERR_CUDA: return "LIME_ERR_CUDA";
+        case LIME_ERR_WORKSPACE: return "LIME_ERR_WORKSPACE";
+        default: return "LIME_ERR_UNKNOWN";
+    }
+}
+
+const char* lime_last_error(void) { return g_last_error; }
+
+lime_status lime_device_check(void) { return check_device(); }
+
+int lime_num_sms(void) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return device_num_sms();
+}
+
+void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread) {
+    g_override.grid_ctas = grid_ctas > 0 ? grid_ctas : 0;
+    g_override.block_threads = block_threads > 0 ? block_threads : 0;
+    g_override.per_thread = per_thread > 0 ? per_thread : 0;
+}
+
+// ============================================================================== N-Body
+size_t lime_map_nbody_workspace_bytes(int64_t n_src, int64_t tgt_count) {
+    if (n_src < 0 || tgt_count < 0) return 0;
+    return nbody::workspace_bytes(n_src, tgt_count);
+}
+
+int lime_nbody_splits(int64_t n_src) { return n_src < 0 ? 0 : nbody::splits(n_src); }
+
+lime_status lime_map_nbody(const float* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,
+                           float eps2, float* accel, void* ws, size_t ws_bytes, void* stream) {
+    if (n_src < 0 || tgt_begin < 0 || tgt_count < 0 || tgt_begin > n_src || tgt_count > n_src - tgt_begin)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody: shard [%lld, %lld+%lld) outside [0, %lld)",
+                    (long long)tgt_begin, (long long)tgt_begin, (long long)tgt_count, (long long)n_src);
+    if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody: eps2 must be finite and >= FLT_MIN (got %g)", (double)eps2);
+    if (tgt_count == 0) return LIME_OK;
+    if (!bodies || !accel || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody: null pointer");
+    if (!aligned16(bodies) || !aligned16(accel) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_nbody: bodies, accel and ws must be 16-byte aligned");
+    if (overlap(accel, tgt_count * 16, bodies, n_src * 16))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody: accel overlaps bodies");
+    if (overlap(ws, ws_bytes, bodies, n_src * 16) || overlap(ws, ws_bytes, accel, tgt_count * 16))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody: workspace overlaps an operand");
+    LIME_TRY(check_device());
+    const size_t need = nbody::workspace_bytes(n_src, tgt_count);
+    if (ws_bytes < need)
+        return fail(LIME_ERR_WORKSPACE, "lime_map_nbody: workspace %zu B < %zu B", ws_bytes, need);
+    return launched(nbody::launch_force(reinterpret_cast<const float4*>(bodies), n_src, tgt_begin, tgt_count, eps2,
+                                        reinterpret_cast<float4*>(accel), ws, static_cast<cudaStream_t>(stream)),
+                    "lime_map_nbody");
+}
+
+lime_status lime_map_nbody_integrate(float* pos, float* vel, const float* accel, int64_t n, float dt, void* stream) {
+    if (n < 0) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_integrate: n < 0");
+    if (!std::isfinite(dt)) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_integrate: dt not finite");
+    if (n == 0) return LIME_OK;
+    if (!pos || !vel || !accel) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_integrate: null pointer");
+    if (!aligned16(pos) || !aligned16(vel) || !aligned16(accel))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_nbody_integrate: operands must be 16-byte aligned");
+    const size_t b = static_cast<size_t>(n) * 16;
+    if (overlap(pos, b, vel, b) || overlap(accel, b, pos, b) || overlap(accel, b, vel, b))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody_integrate: pos, vel and accel must be disjoint");
+    LIME_TRY(check_device());
+    return launched(nbody::launch_integrate(reinterpret_cast<float4*>(pos), reinterpret_cast<float4*>(vel),
+                                            reinterpret_cast<const float4*>(accel), n, dt,
+                                            static_cast<cudaStream_t>(stream)),
+                    "lime_map_nbody_integrate");
+}
+
+// ws layout: [pos n*16][vel n*16][accel n*16][nbody workspace]
+size_t lime_nbody_simulate_host_workspace_bytes(int64_t n) {
+    if (n < 0) return 0;
+    return static_cast<size_t>(n) * 48 + nbody::workspace_bytes(n, n);
+}
+
+lime_status lime_nbody_simulate_host(float* h_pos, float* h_vel, int64_t n, int32_t steps, float eps2, float dt,
+                                     void* ws, size_t ws_bytes, void* stream) {
+    if (n < 0 || steps < 0) return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: n or steps < 0");
+    if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f) || !std::isfinite(dt))
+        return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: bad eps2 or dt");
+    if (n == 0) return LIME_OK;
+    if (!h_pos || !h_vel || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: null pointer");
+    if (!aligned16(ws)) return fail(LIME_ERR_MISALIGNED, "lime_nbody_simulate_host: ws must be 16-byte aligned");
+    const size_t b = static_cast<size_t>(n) * 16;
+    if (overlap(h_pos, b, h_vel, b)) return fail(LIME_ERR_ALIASING, "lime_nbody_simulate_host: h_pos overlaps h_vel");
+    LIME_TRY(check_device());
+    if (ws_bytes < lime_nbody_simulate_host_workspace_bytes(n))
+        return fail(LIME_ERR_WORKSPACE, "lime_nbody_simulate_host: workspace too small");
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    char* w = static_cast<char*>(ws);
+    float4* d_pos = reinterpret_cast<float4*>(w);
+    float4* d_vel = reinterpret_cast<float4*>(w + b);
+    float4* d_acc = reinterpret_cast<float4*>(w + 2 * b);
+    void* d_ws = w + 3 * b;
+    cudaError_t e = cudaMemcpyAsync(d_pos, h_pos, b, cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(d_vel, h_vel, b, cudaMemcpyHostToDevice, s);
+    for (int32_t k = 0; k < steps && e == cudaSuccess; ++k) {
+        e = nbody::launch_force(d_pos, n, 0, n, eps2, d_acc, d_ws, s);
+        if (e == cudaSuccess) e = nbody::launch_integrate(d_pos, d_vel, d_acc, n, dt, s);
+    }
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_pos, d_pos, b, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_vel, d_vel, b, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    return launched(e, "lime_nbody_simulate_host");
+}
+
+// ======================================================================= Black-Scholes
+static lime_status bs_validate(const char* fn, const float* S, const float* X, const float* T, int64_t n,
+                               float r, float sigma) {
+    if (n < 0) return fail(LIME_ERR_INVALID_ARG, "%s: n < 0", fn);
+    if (!std::isfinite(r) || !(sigma > 0.f) || !std::isfinite(sigma))
+        return fail(LIME_ERR_INVALID_ARG, "%s: r must be finite and sigma finite and > 0", fn);
+    if (n > 0 && (!S || !X || !T)) return fail(LIME_ERR_INVALID_ARG, "%s: null input", fn);
+    if (n > 0 && (!aligned16(S) || !aligned16(X) || !aligned16(T)))
+        return fail(LIME_ERR_MISALIGNED, "%s: S, X, T must be 16-byte aligned", fn);
+    return LIME_OK;
+}
+
+lime_status lime_map_blackscholes(const float* S, const float* X, const float* T, int64_t n, float r, float sigma,
+                                  float* call, float* put, void* stream) {
+    LIME_TRY(bs_validate("lime_map_blackscholes", S, X, T, n, r, sigma));
+    if (n == 0) return LIME_OK;
+    if (!call || !put) return fail(LIME_ERR_INVALID_ARG, "lime_map_blackscholes: null output");
+    if (!aligned16(call) || !aligned16(put))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_blackscholes: call, put must be 16-byte aligned");
+    const size_t b = static_cast<size_t>(n) * 4;
+    for (const void* in : {static_cast<const void*>(S), static_cast<const void*>(X), static_cast<const void*>(T)})
+        if (overlap(call, b, in, b) || overlap(put, b, in, b))
+            return fail(LIME_ERR_ALIASING, "lime_map_blackscholes: an output overlaps an input");
+    if (overlap(call, b, put, b)) return fail(LIME_ERR_ALIASING, "lime_map_blackscholes: call overlaps put");
+    LIME_TRY(check_device());
+    return launched(bs::launch_map(S, X, T, n, r, sigma, call, put, static_cast<cudaStream_t>(stream)),
+                    "lime_map_blackscholes");
+}
+
+lime_status lime_map_reduce_blackscholes_sum(const float* S, const float* X, const float* T, int64_t n, float r,
+                                             float sigma, double* sums, void* ws, size_t ws_bytes, void* stream) {
+    LIME_TRY(bs_validate("lime_map_reduce_blackscholes_sum", S, X, T, n, r, sigma));
+    if (!sums || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_reduce_blackscholes_sum: null sums or ws");
+    if (!aligned16(ws)) return fail(LIME_ERR_MISALIGNED, "lime_map_reduce_blackscholes_sum: ws must be 16-byte aligned");
+    const size_t b = static_cast<size_t>(n) * 4;
+    for (const void* in : {static_cast<const void*>(S), static_cast<const void*>(X), static_cast<const void*>(T)})
+        if (overlap(sums, 16, in, b) || overlap(ws, ws_bytes, in, b))
+            return fail(LIME_ERR_ALIASING, "lime_map_reduce_blackscholes_sum: sums/ws overlap an input");
+    if (overlap(sums, 16, ws, ws_bytes)) return fail(LIME_ERR_ALIASING, "lime_map_reduce_blackscholes_sum: sums overlaps ws");
+    LIME_TRY(check_device());
+    if (ws_bytes < red::kWorkspaceBytes)
+        return fail(LIME_ERR_WORKSPACE, "lime_map_reduce_blackscholes_sum: workspace %zu B < %zu B", ws_bytes,
+                    red::kWorkspaceBytes);
+    return launched(bs::launch_map_reduce(S, X, T, n, r, sigma, sums, ws, static_cast<cudaStream_t>(stream)),
+                    "lime_map_reduce_blackscholes_sum");
+}
+
+// ========================================================================== Mandelbrot
+size_t lime_mandelbrot_workspace_bytes(void) { return mandel::kWorkspaceBytes; }
+
+lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first, int32_t row_stride,
+                                int32_t row_count, float x0, float y0, float dx, float dy, int32_t max_iter,
+                                int32_t* counts, void* ws, size_t ws_bytes, void* stream) {
+    if (width <= 0 || height <= 0 || row_stride < 1 || row_count < 0 || row_first < 0 || row_first >= height ||
+        max_iter < 0)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_mandelbrot: bad geometry or max_iter");
+    if (row_count > 0 && static_cast<int64_t>(row_first) + static_cast<int64_t>(row_count - 1) * row_stride >= height)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_mandelbrot: addressed rows exceed height");
+    if (!std::isfinite(x0) || !std::isfinite(y0) || !std::isfinite(dx) || !std::isfinite(dy))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_mandelbrot: non-finite region");
+    if (row_count == 0) return LIME_OK;
+    if (!counts || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_mandelbrot: null pointer");
+    if ((reinterpret_cast<uintptr_t>(counts) & 3u) != 0 || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_mandelbrot: counts must be 4-B and ws 16-B aligned");
+    if (overlap(counts, static_cast<size_t>(row_count) * width * 4, ws, ws_bytes))
+        return fail(LIME_ERR_ALIASING, "lime_map_mandelbrot: counts overlaps ws");
+    LIME_TRY(check_device());
+    if (ws_bytes < mandel::kWorkspaceBytes) return fail(LIME_ERR_WORKSPACE, "lime_map_mandelbrot: workspace too small");
+    return launched(mandel::launch(width, row_first, row_stride, row_count, x0, y0, dx, dy, max_iter, counts, ws,
+                                   static_cast<cudaStream_t>(stream)),
+                    "lime_map_mandelbrot");
+}
+
+// ============================================================================== Matmul
+lime_status lime_map_matmul_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
+                                 void* stream) {
+    if (M < 1 || N < 1 || K < 8 || (K % 8) != 0)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: need M, N >= 1 and K >= 8, K %% 8 == 0");
+    if (M > (1LL << 31) || N > (1LL << 31) || K > (1LL << 31))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: dimension exceeds 2^31");
+    if (!A || !Bt || !C) return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: null pointer");
+    if (!aligned16(A) || !aligned16(Bt) || !aligned16(C))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_matmul_bf16: A, Bt, C must be 16-byte aligned");
+    const size_t cb = static_cast<size_t>(M) * N * 4;
+    if (overlap(C, cb, A, static_cast<size_t>(M) * K * 2) || overlap(C, cb, Bt, static_cast<size_t>(N) * K * 2))
+        return fail(LIME_ERR_ALIASING, "lime_map_matmul_bf16: C overlaps an input");
+    LIME_TRY(check_device());
+    cudaError_t e = gemm::launch_bf16(A, Bt, C, M, N, K, static_cast<cudaStream_t>(stream));
+    if (e == cudaErrorNotSupported) return fail(LIME_ERR_UNSUPPORTED, "lime_map_matmul_bf16: not supported");
+    return launched(e, "lime_map_matmul_bf16");
+}
+
+// ========================================================================== Reductions
+size_t lime_reduce_workspace_bytes(void) { return red::kWorkspaceBytes; }
+
+static lime_status reduce_entry(const char* fn, red::Op op, red::Dt dt, size_t esz, const void* x, int64_t n,
+                                void* out, size_t osz, void* ws, size_t ws_bytes, void* stream) {
+    if (n < 0) return fail(LIME_ERR_INVALID_ARG, "%s: n < 0", fn);
+    if ((n > 0 && !x) || !out || !ws) return fail(LIME_ERR_INVALID_ARG, "%s: null pointer", fn);
+    if ((reinterpret_cast<uintptr_t>(x) % esz) != 0 || (reinterpret_cast<uintptr_t>(out) % osz) != 0 || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "%s: x/out need natural alignment, ws 16-B", fn);
+    const size_t xb = static_cast<size_t>(n) * esz;
+    if (overlap(out, osz, x, xb) || overlap(ws, ws_bytes, x, xb) || overlap(ws, ws_bytes, out, osz))
+        return fail(LIME_ERR_ALIASING, "%s: out/ws overlap", fn);
+    LIME_TRY(check_device());
+    if (ws_bytes < red::kWorkspaceBytes) return fail(LIME_ERR_WORKSPACE, "%s: workspace too small", fn);
+    return launched(red::launch(op, dt, x, n, out, ws, static_cast<cudaStream_t>(stream)), fn);
+}
+
+#define LIME_REDUCE_ENTRY(OPN, OPE, DTN, DTE, T)                                                            \
+    lime_status lime_reduce_##OPN##_##DTN(const T* x, int64_t n, T* out, void* ws, size_t ws_bytes,         \
+                                          void* stream) {                                                   \
+        return reduce_entry("lime_reduce_" #OPN "_" #DTN, OPE, DTE, sizeof(T), x, n, out, sizeof(T), ws,    \
+                            ws_bytes, stream);                                                              \
+    }
+LIME_REDUCE_ENTRY(sum, red::kSum, f32, red::kF32, float)
+LIME_REDUCE_ENTRY(sum, red::kSum, f64, red::kF64, double)
+LIME_REDUCE_ENTRY(sum, red::kSum, i32, red::kI32, int32_t)
+LIME_REDUCE_ENTRY(sum, red::kSum, i64, red::kI64, int64_t)
+LIME_REDUCE_ENTRY(min, red::kMin, f32, red::kF32, float)
+LIME_REDUCE_ENTRY(min, red::kMin, f64, red::kF64, double)
+LIME_REDUCE_ENTRY(min, red::kMin, i32, red::kI32, int32_t)
+LIME_REDUCE_ENTRY(min, red::kMin, i64, red::kI64, int64_t)
+LIME_REDUCE_ENTRY(max, red::kMax, f32, red::kF32, float)
+LIME_REDUCE_ENTRY(max, red::kMax, f64, red::kF64, double)
+LIME_REDUCE_ENTRY(max, red::kMax, i32, red::kI32, int32_t)
+LIME_REDUCE_ENTRY(max, red::kMax, i64, red::kI64, int64_t)
+#undef LIME_REDUCE_ENTRY
+
+}  // extern "C"

@@ -1,0 +1,62 @@
+// kernels.h -- internal launcher interface between abi.cu (validation, C ABI) and the
+// kernel translation units. Not installed; the public contract is include/lime.h.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace lime {
+
+struct LaunchOverride {
+    int grid_ctas = 0;
+    int block_threads = 0;
+    int per_thread = 0;
+};
+const LaunchOverride& launch_override();
+int device_num_sms();
+
+// ------------------------------------------------------------------ N-Body
+namespace nbody {
+constexpr int kChunk = 256;      // two-level accumulation chunk (part of the result's definition)
+constexpr int kMaxSplits = 16;   // split-j partials per target (function of n_src only)
+int64_t chunks_per_split(int64_t n_src);
+int splits(int64_t n_src);
+size_t workspace_bytes(int64_t n_src, int64_t tgt_count);
+cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,
+                         float eps2, float4* accel, void* ws, cudaStream_t stream);
+cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int64_t n, float dt,
+                             cudaStream_t stream);
+}  // namespace nbody
+
+// ----------------------------------------------------------- Black-Scholes
+namespace bs {
+cudaError_t launch_map(const float* S, const float* X, const float* T, int64_t n, float r,
+                       float sigma, float* call, float* put, cudaStream_t stream);
+cudaError_t launch_map_reduce(const float* S, const float* X, const float* T, int64_t n, float r,
+                              float sigma, double* sums, void* ws, cudaStream_t stream);
+}  // namespace bs
+
+// -------------------------------------------------------------- Mandelbrot
+namespace mandel {
+constexpr size_t kWorkspaceBytes = 256;
+cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t row_count,
+                   float x0, float y0, float dx, float dy, int32_t max_iter, int32_t* counts,
+                   void* ws, cudaStream_t stream);
+}  // namespace mandel
+
+// ------------------------------------------------------------------ Matmul
+namespace gemm {
+cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N,
+                        int64_t K, cudaStream_t stream);
+}  // namespace gemm
+
+// -------------------------------------------------------------- Reductions
+namespace red {
+constexpr int kMaxCtas = 148 * 8;
+constexpr size_t kWorkspaceBytes = 256 + 16 * kMaxCtas;   // ticket + up to 16-B partial per CTA
+enum Op { kSum = 0, kMin = 1, kMax = 2 };
+enum Dt { kF32 = 0, kF64 = 1, kI32 = 2, kI64 = 3 };
+cudaError_t launch(Op op, Dt dt, const void* x, int64_t n, void* out, void* ws, cudaStream_t stream);
+}  // namespace red
+
+}  // namespace lime

@@ -1,0 +1,138 @@
+// mandelbrot.cu -- bit-exact Mandelbrot escape-count map (sm_100a).
+//
+// BASELINE.json config 3 (not in the paper; R7). Every multiply/add is an explicit
+// IEEE binary32 round-to-nearest PTX op (mul.rn / add.rn / their .f32x2 packed forms), which
+// the compiler may never contract into FMA and which never flush subnormals -- so the counts
+// equal the oracle's exact binary32 emulation bit for bit.
+//
+// B200 design (DESIGN.md §"Mandelbrot"):
+//  * A5/A6c: each lane iterates TWO horizontally adjacent pixels with packed FMUL2/FADD2
+//    (8 packed ops per pixel pair per iteration instead of 16 scalar ones).
+//  * Branch-free iteration with sticky "alive" predicates; the warp checks __any_sync once
+//    per 16 unrolled iterations, so escaped lanes cost at most 15 extra iterations.
+//  * A1: persistent CTAs pull 16x4-pixel warp tiles from a global atomic queue (dynamic
+//    load balance: escape times vary by 1000x across the frame); the last warp to finish
+//    resets the queue (self-cleaning workspace).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace lime {
+namespace mandel {
+
+constexpr int kTileW = 16;   // pixels per warp tile row (8 lanes x 2 pixels)
+constexpr int kTileH = 4;    // rows per warp tile
+constexpr int kUnroll = 16;
+
+struct Args {
+    int32_t width, row_first, row_stride, row_count;
+    float x0, y0, dx, dy;
+    int32_t max_iter;
+    int32_t* counts;
+    unsigned* queue;   // [0] next tile, [1] warps finished
+    int32_t tiles_x;
+    int64_t ntiles;
+    unsigned total_warps;
+};
+
+struct State {
+    float2 x, y, cx, cy;
+    int n0, n1;
+    bool a0, a1;
+    __device__ __forceinline__ void step() {
+        const float2 xx = mul2(x, x);
+        const float2 yy = mul2(y, y);
+        const float2 s = add2(xx, yy);
+        a0 = a0 && (s.x <= 4.0f);          // test before the update (R7); sticky once escaped
+        a1 = a1 && (s.y <= 4.0f);
+        n0 += a0 ? 1 : 0;
+        n1 += a1 ? 1 : 0;
+        const float2 xy = mul2(x, y);
+        x = add2(sub2(xx, yy), cx);         // x <- (x^2 - y^2) + cx
+        y = add2(add2(xy, xy), cy);         // y <- (xy + xy) + cy
+    }
+};
+
+__global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Args a) {
+    const unsigned lane = lane_id();
+    for (;;) {
+        int64_t tile = 0;
+        if (lane == 0) tile = atomicAdd(a.queue, 1u);
+        tile = __shfl_sync(0xffffffffu, tile, 0);
+        if (tile >= a.ntiles) break;
+        const int32_t tx = static_cast<int32_t>(tile % a.tiles_x);
+        const int32_t ty = static_cast<int32_t>(tile / a.tiles_x);
+        const int32_t col = tx * kTileW + static_cast<int32_t>(lane & 7) * 2;
+        const int32_t k = ty * kTileH + static_cast<int32_t>(lane >> 3);
+        const bool v0 = (col < a.width) && (k < a.row_count);
+        const bool v1 = (col + 1 < a.width) && (k < a.row_count);
+        const int32_t py = a.row_first + min(k, a.row_count - 1) * a.row_stride;
+
+        State st;
+        st.cx = make_float2(add_rn(a.x0, mul_rn(static_cast<float>(col), a.dx)),
+                            add_rn(a.x0, mul_rn(static_cast<float>(col + 1), a.dx)));
+        st.cy = bcast2(add_rn(a.y0, mul_rn(static_cast<float>(py), a.dy)));
+        st.x = make_float2(0.f, 0.f);
+        st.y = make_float2(0.f, 0.f);
+        st.n0 = st.n1 = 0;
+        st.a0 = st.a1 = true;
+
+        int32_t it = 0;
+        while (it + kUnroll <= a.max_iter) {
+#pragma unroll
+            for (int u = 0; u < kUnroll; ++u) st.step();
+            it += kUnroll;
+            if (!__any_sync(0xffffffffu, st.a0 || st.a1)) break;
+        }
+        if (__any_sync(0xffffffffu, st.a0 || st.a1)) {
+            for (; it < a.max_iter; ++it) st.step();
+        }
+        int32_t* row = a.counts + static_cast<int64_t>(k) * a.width;
+        if (v0) row[col] = st.n0;
+        if (v1) row[col + 1] = st.n1;
+    }
+    // Self-cleaning queue: the last warp out resets both counters for the next launch.
+    if (lane == 0) {
+        __threadfence();
+        if (atomicAdd(a.queue + 1, 1u) == a.total_warps - 1) {
+            a.queue[0] = 0u;
+            a.queue[1] = 0u;
+        }
+    }
+}
+
+cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t row_count, float x0,
+                   float y0, float dx, float dy, int32_t max_iter, int32_t* counts, void* ws,
+                   cudaStream_t stream) {
+    if (row_count == 0 || width == 0) return cudaSuccess;
+    Args a;
+    a.width = width;
+    a.row_first = row_first;
+    a.row_stride = row_stride;
+    a.row_count = row_count;
+    a.x0 = x0;
+    a.y0 = y0;
+    a.dx = dx;
+    a.dy = dy;
+    a.max_iter = max_iter;
+    a.counts = counts;
+    a.queue = static_cast<unsigned*>(ws);
+    a.tiles_x = ceil_div<int32_t>(width, kTileW);
+    a.ntiles = static_cast<int64_t>(a.tiles_x) * ceil_div<int32_t>(row_count, kTileH);
+    int grid = launch_override().grid_ctas;
+    if (grid <= 0) {
+        static int per_sm = 0;
+        if (per_sm == 0) {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mandel_kernel, 256, 0);
+            if (per_sm <= 0) per_sm = 1;
+        }
+        grid = per_sm * device_num_sms();
+        const int64_t need = ceil_div<int64_t>(a.ntiles, 8);
+        if (need < grid) grid = static_cast<int>(need);
+    }
+    a.total_warps = static_cast<unsigned>(grid) * 8u;
+    mandel_kernel<<<grid, 256, 0, stream>>>(a);
+    return cudaGetLastError();
+}
+
+}  // namespace mandel
+}  // namespace lime

@@ -1,0 +1,337 @@
+// nbody.cu -- all-pairs N-Body force map and integrator for sm_100a.
+//
+// The paper's workload (PAPER.md L106-114 task graph; L108-112 float[[][4]] particles;
+// L156-158 the map of computeParticleForces over `particles`; L173-174 "n^2 force
+// calculation"). Formula: DESIGN.md R1-R3 (Plummer-softened gravity, G = 1, acceleration).
+//
+// B200 design (DESIGN.md §"N-Body force map"):
+//  * A4 (local-memory tiling, L234-241): the broadcast operand (all sources j) is staged
+//    into shared memory as 16-KB tiles by 1-D TMA bulk copies (cp.async.bulk + mbarrier
+//    complete_tx), double-buffered; every lane reads the same j (LDS.128 broadcast: no bank
+//    conflicts by construction, the B200 form of the paper's conflict padding, L241-255).
+//  * A5 (private memory, L228-233): R targets per thread live in registers (register
+//    blocking), so each staged source feeds R interactions.
+//  * A6a: per interaction 12 FP32 lane-ops + 1 MUFU.RSQ; with R even, pairs of targets use
+//    packed FADD2/FFMA2/FMUL2 (6 issue slots per interaction); bit-identical to the scalar
+//    variant (each half is one IEEE op in the same order).
+//  * A1 (L201-208): results are independent of the launch configuration: a target's sum
+//    order is fixed by the 256-body chunk grid and the split count, both functions of n_src.
+//  * A8 (split-j): S = splits(n_src) source ranges are processed by separate CTAs; the last
+//    CTA of a target tile to finish (atomic ticket) adds the S partials in s order --
+//    one launch, deterministic, self-resetting counters.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace lime {
+namespace nbody {
+
+constexpr int kTileJ = 1024;   // sources per shared-memory stage (16 KB)
+static_assert(kTileJ % kChunk == 0, "stage must hold whole chunks");
+
+int64_t chunks_per_split(int64_t n_src) {
+    const int64_t chunks = ceil_div<int64_t>(n_src, kChunk);
+    return chunks == 0 ? 1 : ceil_div<int64_t>(chunks, kMaxSplits);
+}
+int splits(int64_t n_src) {
+    const int64_t chunks = ceil_div<int64_t>(n_src, kChunk);
+    if (chunks <= 1) return 1;
+    return static_cast<int>(ceil_div<int64_t>(chunks, chunks_per_split(n_src)));
+}
+
+// workspace: [counters: one u32 per 128-target tile, padded to 256 B][partials: S x count float4]
+static size_t counters_bytes(int64_t tgt_count) {
+    return ((ceil_div<int64_t>(tgt_count, 128) * 4 + 255) / 256) * 256;
+}
+size_t workspace_bytes(int64_t n_src, int64_t tgt_count) {
+    const int S = splits(n_src);
+    if (S == 1) return 256;
+    return counters_bytes(tgt_count) + static_cast<size_t>(S) * static_cast<size_t>(tgt_count) * 16;
+}
+
+struct ForceArgs {
+    const float4* bodies;
+    int64_t n_src;
+    int64_t tgt_begin;
+    int64_t tgt_count;
+    float eps2;
+    float4* accel;
+    float4* partial;      // [S][tgt_count]
+    unsigned* counters;   // [tiles]
+    int splits;
+    int64_t split_len;    // chunks_per_split * kChunk
+};
+
+template <int R, bool kPacked>
+struct Interact;
+
+// Scalar: one target per register slot.
+template <int R>
+struct Interact<R, false> {
+    float px[R], py[R], pz[R];
+    float ax[R], ay[R], az[R];   // split accumulators (sum of chunk partials)
+    float cx[R], cy[R], cz[R];   // chunk partials
+    __device__ __forceinline__ void zero_all() {
+#pragma unroll
+        for (int r = 0; r < R; ++r) ax[r] = ay[r] = az[r] = 0.f;
+    }
+    __device__ __forceinline__ void set(int r, float4 p) { px[r] = p.x; py[r] = p.y; pz[r] = p.z; }
+    __device__ __forceinline__ void chunk_begin() {
+#pragma unroll
+        for (int r = 0; r < R; ++r) cx[r] = cy[r] = cz[r] = 0.f;
+    }
+    __device__ __forceinline__ void chunk_end() {
+#pragma unroll
+        for (int r = 0; r < R; ++r) { ax[r] += cx[r]; ay[r] += cy[r]; az[r] += cz[r]; }
+    }
+    __device__ __forceinline__ void body(const float4 b, const float eps2) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const float dx = b.x - px[r];
+            const float dy = b.y - py[r];
+            const float dz = b.z - pz[r];
+            const float r2 = fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2)));
+            const float inv = rsqrt_approx(r2);
+            const float inv2 = inv * inv;
+            const float s = (b.w * inv) * inv2;           // m_j (r^2 + eps^2)^{-3/2}
+            cx[r] = fmaf(s, dx, cx[r]);
+            cy[r] = fmaf(s, dy, cy[r]);
+            cz[r] = fmaf(s, dz, cz[r]);
+        }
+    }
+    __device__ __forceinline__ float4 result(int r) const { return make_float4(ax[r], ay[r], az[r], 0.f); }
+};
+
+// Packed: targets (2q, 2q+1) share each FFMA2/FADD2/FMUL2; same per-lane op order as scalar.
+template <int R>
+struct Interact<R, true> {
+    static_assert(R % 2 == 0, "packed variant pairs targets");
+    static constexpr int Q = R / 2;
+    float2 px[Q], py[Q], pz[Q];
+    float2 ax[Q], ay[Q], az[Q];
+    float2 cx[Q], cy[Q], cz[Q];
+    __device__ __forceinline__ void zero_all() {
+#pragma unroll
+        for (int q = 0; q < Q; ++q) ax[q] = ay[q] = az[q] = make_float2(0.f, 0.f);
+    }
+    __device__ __forceinline__ void set(int r, float4 p) {
+        if (r & 1) { px[r >> 1].y = p.x; py[r >> 1].y = p.y; pz[r >> 1].y = p.z; }
+        else       { px[r >> 1].x = p.x; py[r >> 1].x = p.y; pz[r >> 1].x = p.z; }
+    }
+    __device__ __forceinline__ void chunk_begin() {
+#pragma unroll
+        for (int q = 0; q < Q; ++q) cx[q] = cy[q] = cz[q] = make_float2(0.f, 0.f);
+    }
+    __device__ __forceinline__ void chunk_end() {
+#pragma unroll
+        for (int q = 0; q < Q; ++q) { ax[q] = add2(ax[q], cx[q]); ay[q] = add2(ay[q], cy[q]); az[q] = add2(az[q], cz[q]); }
+    }
+    __device__ __forceinline__ void body(const float4 b, const float eps2) {
+        const float2 e2 = bcast2(eps2);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+            const float2 dx = sub2(bcast2(b.x), px[q]);
+            const float2 dy = sub2(bcast2(b.y), py[q]);
+            const float2 dz = sub2(bcast2(b.z), pz[q]);
+            const float2 r2 = fma2(dx, dx, fma2(dy, dy, fma2(dz, dz, e2)));
+            const float2 inv = make_float2(rsqrt_approx(r2.x), rsqrt_approx(r2.y));
+            const float2 inv2 = mul2(inv, inv);
+            const float2 s = mul2(mul2(bcast2(b.w), inv), inv2);
+            cx[q] = fma2(s, dx, cx[q]);
+            cy[q] = fma2(s, dy, cy[q]);
+            cz[q] = fma2(s, dz, cz[q]);
+        }
+    }
+    __device__ __forceinline__ float4 result(int r) const {
+        const int q = r >> 1;
+        return (r & 1) ? make_float4(ax[q].y, ay[q].y, az[q].y, 0.f) : make_float4(ax[q].x, ay[q].x, az[q].x, 0.f);
+    }
+};
+
+template <int BLOCK, int R, bool kPacked>
+__global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ ForceArgs a) {
+    __shared__ __align__(128) float4 sbuf[2][kTileJ];
+    __shared__ __align__(8) uint64_t full[2];
+    __shared__ int s_last;
+
+    const int tile = blockIdx.x;
+    const int split = blockIdx.y;
+    const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * R);
+
+    // ---- this thread's targets (A3: one 128-bit read-only load each, coalesced)
+    Interact<R, kPacked> it;
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        valid[r] = t < a.tgt_count;
+        const int64_t i = a.tgt_begin + (valid[r] ? t : a.tgt_count - 1);
+        it.set(r, __ldg(a.bodies + i));
+    }
+    it.zero_all();
+
+    // ---- this split's source range [j0, j1)
+    const int64_t j0 = static_cast<int64_t>(split) * a.split_len;
+    const int64_t j1 = min(a.n_src, j0 + a.split_len);
+    const int ntiles = static_cast<int>(ceil_div<int64_t>(j1 - j0, kTileJ));
+
+    if (threadIdx.x == 0) {
+        mbar_init(&full[0], 1);
+        mbar_init(&full[1], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    auto issue = [&](int t) {
+        const int64_t base = j0 + static_cast<int64_t>(t) * kTileJ;
+        const uint32_t bytes = static_cast<uint32_t>(mn<int64_t>(kTileJ, j1 - base)) * 16u;
+        mbar_arrive_expect_tx(&full[t & 1], bytes);
+        bulk_g2s(sbuf[t & 1], a.bodies + base, bytes, &full[t & 1]);
+    };
+    if (threadIdx.x == 0) {
+        issue(0);
+        if (ntiles > 1) issue(1);
+    }
+
+    const float eps2 = a.eps2;
+    for (int t = 0; t < ntiles; ++t) {
+        mbar_wait(&full[t & 1], (t >> 1) & 1);
+        const float4* sb = sbuf[t & 1];
+        const int len = static_cast<int>(mn<int64_t>(kTileJ, j1 - (j0 + static_cast<int64_t>(t) * kTileJ)));
+        for (int c0 = 0; c0 < len; c0 += kChunk) {
+            const int c1 = min(len, c0 + kChunk);
+            it.chunk_begin();
+            if (c1 - c0 == kChunk) {
+#pragma unroll 4
+                for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
+            } else {
+                for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+            }
+            it.chunk_end();
+        }
+        __syncthreads();                            // every lane is done reading this stage
+        if (threadIdx.x == 0 && t + 2 < ntiles) issue(t + 2);
+    }
+
+    // ---- output (A7: float4 stores) / split combine (A8)
+    if (a.splits == 1) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+            if (valid[r]) a.accel[t] = it.result(r);
+        }
+        return;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        if (valid[r]) __stcg(a.partial + static_cast<int64_t>(split) * a.tgt_count + t, it.result(r));
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned prev = atomicAdd(a.counters + tile, 1u);
+        s_last = (prev == static_cast<unsigned>(a.splits - 1));
+    }
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        if (!valid[r]) continue;
+        float4 acc = __ldcg(a.partial + t);
+        for (int s = 1; s < a.splits; ++s) {
+            const float4 p = __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
+            acc.x += p.x; acc.y += p.y; acc.z += p.z;
+        }
+        acc.w = 0.f;
+        a.accel[t] = acc;
+    }
+    if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
+}
+
+template <int BLOCK, int R>
+static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
+    constexpr bool kPacked = (R % 2 == 0);
+    const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
+    dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
+    force_kernel<BLOCK, R, kPacked><<<grid, BLOCK, 0, stream>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,
+                         float eps2, float4* accel, void* ws, cudaStream_t stream) {
+    if (tgt_count == 0) return cudaSuccess;
+    ForceArgs a;
+    a.bodies = bodies;
+    a.n_src = n_src;
+    a.tgt_begin = tgt_begin;
+    a.tgt_count = tgt_count;
+    a.eps2 = eps2;
+    a.accel = accel;
+    a.splits = splits(n_src);
+    a.split_len = chunks_per_split(n_src) * kChunk;
+    a.counters = static_cast<unsigned*>(ws);
+    a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
+
+    const LaunchOverride& ov = launch_override();
+    int block = ov.block_threads, R = ov.per_thread;
+    if (block == 0 || R == 0) {
+        // Automatic: the largest target tile that still gives >= 4 CTAs per SM of work items.
+        const int64_t want = 4LL * device_num_sms();
+        const int cand[][2] = {{256, 4}, {256, 2}, {128, 2}, {128, 1}};
+        int pick = 3;
+        for (int k = 0; k < 4; ++k) {
+            const int64_t items = ceil_div<int64_t>(tgt_count, cand[k][0] * cand[k][1]) * a.splits;
+            if (items >= want) { pick = k; break; }
+        }
+        if (block == 0) block = cand[pick][0];
+        if (R == 0) R = cand[pick][1];
+    }
+    if (block == 256) {
+        switch (R) {
+            case 1: return launch_one<256, 1>(a, stream);
+            case 2: return launch_one<256, 2>(a, stream);
+            case 4: return launch_one<256, 4>(a, stream);
+            case 8: return launch_one<256, 8>(a, stream);
+        }
+    } else if (block == 128) {
+        switch (R) {
+            case 1: return launch_one<128, 1>(a, stream);
+            case 2: return launch_one<128, 2>(a, stream);
+            case 4: return launch_one<128, 4>(a, stream);
+            case 8: return launch_one<128, 8>(a, stream);
+        }
+    }
+    return cudaErrorInvalidConfiguration;
+}
+
+// ------------------------------------------------------------------------ integrator (A9)
+__global__ void __launch_bounds__(256) integrate_kernel(float4* __restrict__ pos, float4* __restrict__ vel,
+                                                        const float4* __restrict__ accel, int64_t n, float dt) {
+    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const float4 a = ld_stream_f4(accel + i);
+        float4 v = vel[i];
+        float4 p = pos[i];
+        v.x = fmaf(a.x, dt, v.x);
+        v.y = fmaf(a.y, dt, v.y);
+        v.z = fmaf(a.z, dt, v.z);
+        p.x = fmaf(v.x, dt, p.x);
+        p.y = fmaf(v.y, dt, p.y);
+        p.z = fmaf(v.z, dt, p.z);
+        vel[i] = v;
+        pos[i] = p;
+    }
+}
+
+cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int64_t n, float dt,
+                             cudaStream_t stream) {
+    if (n == 0) return cudaSuccess;
+    int grid = launch_override().grid_ctas;
+    if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(n, 256), 8LL * device_num_sms()));
+    integrate_kernel<<<grid, 256, 0, stream>>>(pos, vel, accel, n, dt);
+    return cudaGetLastError();
+}
+
+}  // namespace nbody
+}  // namespace lime

@@ -1,0 +1,106 @@
+"""Multi-GPU partitioning of the map index space (BASELINE.json north_star:
+"work is partitioned ... by splitting the map's output index space per GPU").
+
+One process per GPU; torch.distributed (NCCL over NVLink on the box) is the plumbing:
+  * N-Body (config 5): contiguous equal target shards; each step all-gathers positions
+    (`all_gather_into_tensor`, the one real exchange step of the path), runs the force map on
+    the local targets against all sources, then the local integrator. Forces are bit-identical
+    to the single-GPU run because the per-target summation order depends on n_src only.
+  * Black-Scholes fused sums (config 2): contiguous option shards, one `all_reduce` (sum) of the
+    per-GPU fp64 partials.
+  * Mandelbrot (config 3): cyclic rows (row r -> rank r mod P), no collective.
+  * Matmul (config 4): contiguous row blocks of C, no collective.
+
+The step functions take the map/integrator callables as parameters so the partition and
+exchange logic can be exercised on CPU (gloo) in tests; the product binds them to the CUDA ABI.
+"""
+from __future__ import annotations
+
+from typing import Callable
+
+import torch
+import torch.distributed as dist
+
+
+def shard_range(n: int, rank: int, world: int) -> tuple[int, int]:
+    """Contiguous block shard [begin, begin + count) of n elements (balanced to +-1)."""
+    base, rem = divmod(n, world)
+    begin = rank * base + min(rank, rem)
+    return begin, base + (1 if rank < rem else 0)
+
+
+def cyclic_rows(height: int, rank: int, world: int) -> tuple[int, int, int]:
+    """Cyclic row shard for Mandelbrot: (row_first, row_stride, row_count)."""
+    return rank, world, len(range(rank, height, world))
+
+
+class NBodySim:
+    """Sharded N-Body simulation state (positions+mass and velocities of the local shard).
+
+    force_fn(pos_full, tgt_begin, tgt_count, eps2, out) fills out[tgt_count][4];
+    integrate_fn(pos, vel, accel, dt) updates pos/vel in place.
+    """
+
+    def __init__(self, bodies_full: torch.Tensor, eps2: float, dt: float, device,
+                 force_fn: Callable | None = None, integrate_fn: Callable | None = None,
+                 group=None):
+        self.group = group
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        n = bodies_full.shape[0]
+        if n % self.world:
+            raise ValueError("n must be divisible by the number of ranks (equal all-gather shards)")
+        self.n = n
+        self.count = n // self.world
+        self.begin = self.rank * self.count
+        self.eps2, self.dt = eps2, dt
+        self.device = torch.device(device)
+        self.pos = bodies_full[self.begin:self.begin + self.count].to(self.device).contiguous()
+        self.vel = torch.zeros_like(self.pos)
+        self.pos_full = torch.empty((n, 4), dtype=torch.float32, device=self.device)
+        self.accel = torch.empty_like(self.pos)
+        if force_fn is None or integrate_fn is None:
+            import paper_conf_pldi_dubachcrbf12_b200 as lime
+            force_fn = force_fn or (lambda p, b, c, e, out: lime.map_nbody(p, e, b, c, out=out))
+            integrate_fn = integrate_fn or lime.map_nbody_integrate
+        self.force_fn, self.integrate_fn = force_fn, integrate_fn
+
+    def gather(self):
+        if self.world == 1:
+            self.pos_full.copy_(self.pos)
+        else:
+            dist.all_gather_into_tensor(self.pos_full, self.pos, group=self.group)
+
+    def step(self):
+        """One task-graph pass: exchange, force map, integrate."""
+        self.gather()
+        self.force_fn(self.pos_full, self.begin, self.count, self.eps2, self.accel)
+        self.integrate_fn(self.pos, self.vel, self.accel, self.dt)
+
+    def step_host(self, h_pos: torch.Tensor, h_vel: torch.Tensor):
+        """End-to-end step from host (pinned) shard state: H2D, step, D2H."""
+        self.pos.copy_(h_pos, non_blocking=True)
+        self.vel.copy_(h_vel, non_blocking=True)
+        self.step()
+        h_pos.copy_(self.pos, non_blocking=True)
+        h_vel.copy_(self.vel, non_blocking=True)
+
+    def momentum(self) -> torch.Tensor:
+        """Global sum of m v over all ranks (all_reduce), float64 [3]."""
+        m = self.pos[:, 3:4].double()
+        p = (m * self.vel[:, :3].double()).sum(0)
+        if self.world > 1:
+            dist.all_reduce(p, group=self.group)
+        return p
+
+
+def blackscholes_total(S, X, T, r: float, sigma: float, fused_fn: Callable | None = None, group=None):
+    """Global (sum call, sum put) over the option shards of all ranks: local fused map+reduce,
+    then one all_reduce of the two fp64 partials."""
+    if fused_fn is None:
+        import paper_conf_pldi_dubachcrbf12_b200 as lime
+        fused_fn = lime.map_reduce_blackscholes_sum
+    sums = fused_fn(S, X, T, r, sigma)
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(sums, group=group)
+    return sums

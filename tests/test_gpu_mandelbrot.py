@@ -1,0 +1,50 @@
+"""GPU parity: Mandelbrot escape counts, bit-exact vs the oracle's binary32 emulation."""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from testutil import golden
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("W,H,max_iter", [(256, 256, 256), (1000, 37, 100), (17, 9, 1), (64, 64, 0), (333, 200, 1024)])
+def test_small_frames_bit_exact(lime, W, H, max_iter):
+    dx, dy = 3.0 / W, 3.0 / H
+    gpu = lime.map_mandelbrot(W, H, -2.0, -1.5, dx, dy, max_iter).cpu().numpy()
+    ref = oracle.mandelbrot(W, H, 0, 1, H, -2.0, -1.5, dx, dy, max_iter)
+    assert np.array_equal(gpu, ref)
+
+
+def test_hand_checked_points(lime):
+    g = golden("mandelbrot_points.json")
+    for cx, cy, n in g["points"]:
+        out = lime.map_mandelbrot(1, 1, float(np.float32(cx)), float(np.float32(cy)), 0.0, 0.0, g["max_iter"])
+        assert int(out.item()) == n, (cx, cy)
+
+
+def test_cyclic_shards(lime):
+    W = H = 512
+    d = 3.0 / 512
+    full = lime.map_mandelbrot(W, H, -2.0, -1.5, d, d, 300).cpu()
+    for P in (2, 3, 8):
+        for r in range(P):
+            sh = lime.map_mandelbrot(W, H, -2.0, -1.5, d, d, 300, row_first=r, row_stride=P).cpu()
+            assert torch.equal(sh, full[r::P])
+
+
+def test_full_frame_config3(lime):
+    f = golden("mandelbrot_points.json")["frame"]
+    W, H = f["width"], f["height"]
+    gpu = lime.map_mandelbrot(W, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"]).cpu().numpy()
+    assert int(gpu.sum(dtype=np.int64)) == f["checksum"]
+    assert np.array_equal(gpu[1:4096], gpu[8191:4096:-1])            # mirror symmetry
+    rows = np.random.default_rng(3).choice(H, 48, replace=False)
+    for r in rows:
+        ref = oracle.mandelbrot(W, H, int(r), 1, 1, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"])
+        assert np.array_equal(gpu[r], ref[0]), r
+    again = lime.map_mandelbrot(W, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"]).cpu().numpy()
+    assert np.array_equal(gpu, again)

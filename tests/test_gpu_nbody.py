@@ -1,0 +1,123 @@
+"""GPU parity: N-Body force map and integrator vs the oracle (through the C ABI)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_pldi_dubachcrbf12_b200 import inputs
+from testutil import NBODY_RTOL, nbody_rel_err
+
+pytestmark = pytest.mark.gpu
+EPS2 = np.float32(1e-4)
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 31, 33, 255, 256, 257, 1000, 4096, 4097])
+def test_force_matches_oracle(lime, n):
+    b = inputs.nbody_bodies(n, seed=100 + n)
+    acc = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    ref, mag = oracle.nbody_accel(b, EPS2, with_mag=True)
+    err = nbody_rel_err(acc, ref, mag)
+    assert err.max() <= NBODY_RTOL, (n, err.max())
+    assert np.all(acc[:, 3] == 0.0)
+
+
+def test_single_body_and_self_term(lime):
+    b = np.array([[0.25, -0.5, 0.75, 3.0]], dtype=np.float32)
+    assert np.all(lime.map_nbody(_dev(b), 1e-4).cpu().numpy() == 0.0)
+
+
+def test_shards_are_slices_and_launch_independent(lime):
+    n = 4097
+    b = _dev(inputs.nbody_bodies(n, seed=7))
+    full = lime.map_nbody(b, float(EPS2)).cpu()
+    for begin, count in [(0, 1), (1, 1000), (2048, 2049), (4000, 97), (17, 0)]:
+        part = lime.map_nbody(b, float(EPS2), begin, count).cpu()
+        assert torch.equal(part, full[begin:begin + count])
+    for block in (128, 256):
+        for R in (1, 2, 4, 8):
+            with lime.launch_override(block_threads=block, per_thread=R):
+                alt = lime.map_nbody(b, float(EPS2)).cpu()
+            assert torch.equal(alt, full), (block, R)
+
+
+def test_p_way_sharding_bit_identical(lime):
+    n = 1 << 14
+    b = _dev(inputs.nbody_bodies(n, seed=8))
+    full = lime.map_nbody(b, float(EPS2)).cpu()
+    for P in (2, 4, 8):
+        parts = [lime.map_nbody(b, float(EPS2), r * n // P, n // P).cpu() for r in range(P)]
+        assert torch.equal(torch.cat(parts), full)
+
+
+def test_momentum_and_determinism(lime):
+    for n in (4096, 16384):
+        b = inputs.nbody_bodies(n, seed=9)
+        bd = _dev(b)
+        a1 = lime.map_nbody(bd, float(EPS2))
+        a2 = lime.map_nbody(bd, float(EPS2))
+        assert torch.equal(a1, a2)                                  # run-to-run bit identical
+        a = a1.cpu().numpy()[:, :3].astype(np.float64)
+        m = b[:, 3].astype(np.float64)
+        P = (m[:, None] * a).sum(0)
+        assert np.linalg.norm(P) <= 1e-6 * (m * np.linalg.norm(a, axis=1)).sum()
+        assert torch.equal(bd.cpu(), torch.from_numpy(b))          # input untouched (L139-143)
+
+
+def test_config5_sampled_targets(lime):
+    n = 1 << 20
+    b = inputs.nbody_bodies(n, seed=5)
+    acc = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    rows = np.random.default_rng(0).choice(n, 256, replace=False)
+    rows = np.concatenate([rows, [0, n - 1]])
+    ref, mag = oracle.nbody_accel_rows(b, EPS2, rows, threads=8)
+    err = nbody_rel_err(acc[rows], ref, mag)
+    assert err.max() <= NBODY_RTOL, err.max()
+
+
+def test_config5_sharded_launch_matches_full(lime):
+    # the launch bench.py times at P = 8: 2^17 targets against 2^20 sources
+    n, P = 1 << 20, 8
+    b = _dev(inputs.nbody_bodies(n, seed=5))
+    for r in (0, 5):
+        part = lime.map_nbody(b, float(EPS2), r * n // P, n // P)
+        full_slice = lime.map_nbody(b, float(EPS2), r * n // P, 1024)
+        assert torch.equal(part[:1024], full_slice)
+
+
+def test_integrator_one_step(lime):
+    n = 3001
+    b = inputs.nbody_bodies(n, seed=12)
+    vel = (inputs.nbody_bodies(n, seed=13) * np.float32(0.1)).astype(np.float32)
+    vel[:, 3] = 0
+    acc = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    pos_d, vel_d, acc_d = _dev(b), _dev(vel), _dev(acc)
+    lime.map_nbody_integrate(pos_d, vel_d, acc_d, 1e-3)
+    p_ref, v_ref = oracle.nbody_integrate(b, vel, acc, np.float32(1e-3))
+    np.testing.assert_allclose(vel_d.cpu().numpy(), v_ref, rtol=0, atol=2e-7 * np.abs(v_ref).max() + 1e-12)
+    np.testing.assert_allclose(pos_d.cpu().numpy(), p_ref, rtol=0, atol=2e-7)
+    assert np.array_equal(pos_d.cpu().numpy()[:, 3], b[:, 3])     # mass carried
+
+
+def test_simulate_host_matches_device_path(lime):
+    n, steps = 2048, 3
+    b = inputs.nbody_bodies(n, seed=14)
+    h_pos = torch.from_numpy(b.copy()).pin_memory()
+    h_vel = torch.zeros((n, 4), dtype=torch.float32).pin_memory()
+    lime.nbody_simulate_host(h_pos, h_vel, steps, 1e-4, 1e-3)
+    pos, vel = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    for _ in range(steps):
+        a = lime.map_nbody(pos, 1e-4)
+        lime.map_nbody_integrate(pos, vel, a, 1e-3)
+    assert torch.equal(h_pos, pos.cpu()) and torch.equal(h_vel, vel.cpu())
+
+
+def test_errors_surface_as_exceptions(lime):
+    b = _dev(inputs.nbody_bodies(16, seed=1))
+    with pytest.raises(lime.LimeError, match="INVALID_ARG"):
+        lime.map_nbody(b, 0.0)
+    with pytest.raises(lime.LimeError, match="INVALID_ARG"):
+        lime.map_nbody(b, 1e-4, 10, 7)
