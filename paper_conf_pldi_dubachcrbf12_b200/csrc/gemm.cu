@@ -1,7 +1,288 @@
-// gemm.cu -- placeholder until the tcgen05 kernel lands (next commit).
+// gemm.cu -- dense matrix multiply as a map of dot products on the 5th-gen tensor cores (sm_100a).
+//
+// BASELINE.json config 4 (not in the paper; R8): C[i][j] = sum_k A[i][k] Bt[j][k],
+// A [M][K], Bt [N][K] bf16 (K-major: each output element is the dot product of two contiguous
+// K-vectors), C [M][N] fp32. The only dense contraction of the path, so the only kernel on the
+// tensor cores (north_star).
+//
+// Design (DESIGN.md §"Matmul"): persistent, warp-specialised, one CTA per SM:
+//   warp 0      TMA producer: 2-D tensor-map loads (128B swizzle -- the B200 form of the paper's
+//               bank-conflict padding, L241-255) of A/B K-slices into a STAGES-deep smem ring
+//               (A4: local-memory tiling of the broadcast operand, L234-241)
+//   warp 1      TMEM allocator + single-thread tcgen05.mma issuer (kind::f16, BF16 x BF16 -> FP32,
+//               accumulator in TMEM), tcgen05.commit releases smem stages / publishes accumulators
+//   warps 2..5  epilogue: tcgen05.ld TMEM -> registers -> fp32 C (A7), double-buffered TMEM
+//               accumulators (2 x 256 columns) so the epilogue of tile t overlaps the MMAs of t+1.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include "common.cuh"
 #include "kernels.h"
-namespace lime { namespace gemm {
-cudaError_t launch_bf16(const uint16_t*, const uint16_t*, float*, int64_t, int64_t, int64_t, cudaStream_t) {
-    return cudaErrorNotSupported;
+
+namespace lime {
+namespace gemm {
+
+constexpr int BM = 128;            // UMMA_M (cta_group::1)
+constexpr int BN = 256;            // UMMA_N
+constexpr int BK = 64;             // one 128-byte swizzle atom of bf16
+constexpr int UMMA_K = 16;
+constexpr int STAGES = 4;
+constexpr int kThreads = 192;      // 6 warps
+constexpr uint32_t kStageA = BM * BK * 2;       // 16 KB
+constexpr uint32_t kStageB = BN * BK * 2;       // 32 KB
+constexpr uint32_t kStageBytes = kStageA + kStageB;
+constexpr uint32_t kTmemCols = 512;             // 2 accumulators x 256 fp32 columns
+constexpr int kGroupM = 16;                     // raster: 16 M-blocks share B tiles in L2
+constexpr size_t kSmemBytes = 1024 /*align slack*/ + STAGES * kStageBytes + 256 /*barriers*/;
+
+// ------------------------------------------------------------------ PTX wrappers (sm_100a)
+__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, void* dst, uint64_t* bar, int c0, int c1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+        :: "r"(smem_addr(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_addr(bar))
+        : "memory");
 }
-}}
+__device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
+    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                 :: "r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc) : "memory");
+}
+// 32 lanes x 32 consecutive fp32 columns: thread i gets TMEM lane (quadrant*32 + i), columns c..c+31
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+    uint32_t r[32];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+// UMMA shared-memory descriptor: K-major operand, 128-byte swizzle, 8-row core-matrix groups
+// 1024 B apart (SBO), LBO unused (1), descriptor version 1 (sm_100).
+__device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t saddr) {
+    return static_cast<uint64_t>((saddr >> 4) & 0x3FFF) | (static_cast<uint64_t>(1) << 16) |
+           (static_cast<uint64_t>(1024 >> 4) << 32) | (static_cast<uint64_t>(1) << 46) |
+           (static_cast<uint64_t>(2) << 61);
+}
+// Instruction descriptor: kind::f16, A = B = BF16, D = F32, both K-major, M = BM, N = BN.
+constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(BN >> 3) << 17) |
+                            (static_cast<uint32_t>(BM >> 4) << 24);
+
+struct Params {
+    float* C;
+    int M, N, K;
+    int num_m, num_n, num_k;
+    int num_tiles;
+};
+
+__device__ __forceinline__ void tile_coords(int t, const Params& p, int& mb, int& nb) {
+    const int per_group = kGroupM * p.num_n;
+    const int g = t / per_group;
+    const int first_m = g * kGroupM;
+    const int gm = min(p.num_m - first_m, kGroupM);
+    const int r = t - g * per_group;
+    mb = first_m + r % gm;
+    nb = r / gm;
+}
+
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+            const __grid_constant__ Params p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * kStageBytes);
+    uint64_t* empty = full + STAGES;
+    uint64_t* tfull = empty + STAGES;
+    uint64_t* tempty = tfull + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+
+    if (warp == 0 && lane == 0) {
+        prefetch_tmap(&tmap_a);
+        prefetch_tmap(&tmap_b);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull[a], 1);
+            mbar_init(&tempty[a], 4);     // one arrive per epilogue warp
+        }
+        fence_mbar_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_addr(tmem_slot)), "r"(kTmemCols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        // ----------------------------------------------------------- TMA producer
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
+                int mb, nb;
+                tile_coords(t, p, mb, nb);
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&empty[s], ph ^ 1);
+                    uint8_t* sa = smem + s * kStageBytes;
+                    mbar_arrive_expect_tx(&full[s], kStageBytes);
+                    tma_load_2d(&tmap_a, sa, &full[s], kb * BK, mb * BM);
+                    tma_load_2d(&tmap_b, sa + kStageA, &full[s], kb * BK, nb * BN);
+                    if (++s == STAGES) { s = 0; ph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ----------------------------------------------------------- MMA issuer
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            int local = 0;
+            for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++local) {
+                const int acc = local & 1;
+                mbar_wait(&tempty[acc], ((local >> 1) & 1) ^ 1);
+                tc_fence_after();
+                const uint32_t dtm = tmem_base + static_cast<uint32_t>(acc * BN);
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&full[s], ph);
+                    tc_fence_after();
+                    const uint32_t sa = smem_addr(smem + s * kStageBytes);
+                    const uint32_t sb = sa + kStageA;
+#pragma unroll
+                    for (int k = 0; k < BK / UMMA_K; ++k) {
+                        tc_mma(dtm, smem_desc_sw128(sa + k * UMMA_K * 2), smem_desc_sw128(sb + k * UMMA_K * 2), kIdesc,
+                               (kb | k) != 0);
+                    }
+                    tc_commit(&empty[s]);            // frees this smem stage when the MMAs retire
+                    if (++s == STAGES) { s = 0; ph ^= 1; }
+                }
+                tc_commit(&tfull[acc]);              // accumulator complete
+            }
+        }
+        __syncwarp();
+    } else {
+        // ----------------------------------------------------------- epilogue (warps 2..5)
+        const int quad = warp & 3;                   // TMEM lane quadrant this warp may access
+        const int row_in_tile = quad * 32 + lane;
+        int local = 0;
+        for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++local) {
+            const int acc = local & 1;
+            int mb, nb;
+            tile_coords(t, p, mb, nb);
+            mbar_wait(&tfull[acc], (local >> 1) & 1);
+            tc_fence_after();
+            const int row = mb * BM + row_in_tile;
+            const uint32_t tbase = tmem_base + (static_cast<uint32_t>(quad * 32) << 16) + static_cast<uint32_t>(acc * BN);
+            float* crow = p.C + static_cast<int64_t>(row) * p.N;
+            const bool vec_ok = (p.N & 3) == 0;
+#pragma unroll 1
+            for (int c = 0; c < BN; c += 32) {
+                float v[32];
+                tmem_ld32(tbase + c, v);
+                const int col0 = nb * BN + c;
+                if (row < p.M) {
+                    if (vec_ok && col0 + 32 <= p.N) {
+#pragma unroll
+                        for (int q = 0; q < 8; ++q)
+                            st_stream_f4(reinterpret_cast<float4*>(crow + col0) + q,
+                                         make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < 32; ++q)
+                            if (col0 + q < p.N) crow[col0 + q] = v[q];
+                    }
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&tempty[acc]);
+        }
+    }
+
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 1) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem_base), "r"(kTmemCols) : "memory");
+    }
+}
+
+// ------------------------------------------------------------------ host side
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    if (!fn) {
+        void* ptr = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+    }
+    return fn;
+}
+
+static bool make_map(CUtensorMap* map, const void* base, uint64_t rows, uint64_t K, uint32_t box_rows) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[2] = {K, rows};
+    const cuuint64_t strides[1] = {K * 2};
+    const cuuint32_t box[2] = {static_cast<cuuint32_t>(BK), box_rows};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
+                        cudaStream_t stream) {
+    CUtensorMap ma, mb;
+    if (!make_map(&ma, A, M, K, BM) || !make_map(&mb, Bt, N, K, BN)) return cudaErrorInvalidValue;
+    Params p;
+    p.C = C;
+    p.M = static_cast<int>(M);
+    p.N = static_cast<int>(N);
+    p.K = static_cast<int>(K);
+    p.num_m = static_cast<int>(ceil_div<int64_t>(M, BM));
+    p.num_n = static_cast<int>(ceil_div<int64_t>(N, BN));
+    p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
+    p.num_tiles = p.num_m * p.num_n;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(kSmemBytes));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    int grid = launch_override().grid_ctas;
+    if (grid <= 0) grid = device_num_sms();
+    grid = mn(grid, p.num_tiles);
+    gemm_kernel<<<grid, kThreads, kSmemBytes, stream>>>(ma, mb, p);
+    return cudaGetLastError();
+}
+
+}  // namespace gemm
+}  // namespace lime

@@ -1,9 +1,9 @@
 // mandelbrot.cu -- bit-exact Mandelbrot escape-count map (sm_100a).
 //
-// BASELINE.json config 3 (not in the paper; R7). Every multiply/add is an explicit
-// IEEE binary32 round-to-nearest PTX op (mul.rn / add.rn / their .f32x2 packed forms), which
-// the compiler may never contract into FMA and which never flush subnormals -- so the counts
-// equal the oracle's exact binary32 emulation bit for bit.
+// BASELINE.json config 3 (not in the paper; R7). Every multiply/add is one IEEE
+// binary32 round-to-nearest operation (no contraction, no subnormal flushing), so the counts
+// equal the oracle's exact binary32 emulation bit for bit; tests/test_sass_guards.py checks the
+// compiled SASS keeps it that way.
 //
 // B200 design (DESIGN.md §"Mandelbrot"):
 //  * A5/A6c: each lane iterates TWO horizontally adjacent pixels with packed FMUL2/FADD2
@@ -34,21 +34,27 @@ struct Args {
     unsigned total_warps;
 };
 
+// Every binary32 op is written as ONE fused multiply-add whose extra operand makes it exact:
+//   a*b = fma(a, b, -0),  a+b = fma(a, 1, b),  a-b = fma(b, -1, a)
+// ptxas contracts packed mul.rn/add.rn.f32x2 pairs into FFMA2 even with --fmad=false (observed
+// on CUDA 12.9, see tests/test_sass_guards.py), which changes rounding; an FFMA2 cannot be
+// contracted further, so this spelling keeps one IEEE rounding per operation of R7.
 struct State {
     float2 x, y, cx, cy;
     int n0, n1;
     bool a0, a1;
     __device__ __forceinline__ void step() {
-        const float2 xx = mul2(x, x);
-        const float2 yy = mul2(y, y);
-        const float2 s = add2(xx, yy);
-        a0 = a0 && (s.x <= 4.0f);          // test before the update (R7); sticky once escaped
+        const float2 z = bcast2(-0.0f), one = bcast2(1.0f), mone = bcast2(-1.0f);
+        const float2 xx = fma2(x, x, z);
+        const float2 yy = fma2(y, y, z);
+        const float2 s = fma2(xx, one, yy);          // x^2 + y^2
+        a0 = a0 && (s.x <= 4.0f);                    // test before the update (R7); sticky once escaped
         a1 = a1 && (s.y <= 4.0f);
         n0 += a0 ? 1 : 0;
         n1 += a1 ? 1 : 0;
-        const float2 xy = mul2(x, y);
-        x = add2(sub2(xx, yy), cx);         // x <- (x^2 - y^2) + cx
-        y = add2(add2(xy, xy), cy);         // y <- (xy + xy) + cy
+        const float2 xy = fma2(x, y, z);
+        x = fma2(fma2(yy, mone, xx), one, cx);       // x <- (x^2 - y^2) + cx
+        y = fma2(fma2(xy, one, xy), one, cy);        // y <- (xy + xy) + cy
     }
 };
 

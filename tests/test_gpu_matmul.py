@@ -1,0 +1,70 @@
+"""GPU parity: tcgen05 bf16 matmul (map of dot products) vs the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_pldi_dubachcrbf12_b200 import inputs
+from testutil import MATMUL_RTOL
+
+pytestmark = pytest.mark.gpu
+
+
+def _bf(a_bits):
+    return torch.from_numpy(np.ascontiguousarray(a_bits).view(np.int16)).cuda().view(torch.bfloat16)
+
+
+def _check(C, A, Bt, rows=None, cols=None):
+    if rows is None:
+        ref = oracle.matmul_bf16(A, Bt)
+        mag = np.abs(inputs.bf16_bits_to_f32(A)).astype(np.float64) @ np.abs(inputs.bf16_bits_to_f32(Bt)).astype(np.float64).T
+        err = np.abs(C.astype(np.float64) - ref) / np.maximum(mag, 1e-30)
+        fro = np.linalg.norm(C - ref) / max(np.linalg.norm(ref), 1e-30)
+        return err.max(), fro
+    ref, mag = oracle.matmul_bf16_entries(A, Bt, rows, cols, threads=8)
+    err = np.abs(C[rows, cols].astype(np.float64) - ref) / np.maximum(mag, 1e-30)
+    return err.max(), 0.0
+
+
+@pytest.mark.parametrize("M,N,K", [(128, 256, 64), (1, 1, 8), (33, 47, 72), (300, 520, 200), (256, 512, 1024),
+                                   (1000, 1000, 1000), (8192 // 8, 64, 128), (129, 257, 4104)])
+def test_matmul_small_matches_oracle(lime, M, N, K):
+    A, Bt = inputs.matmul_operands(M, N, K, seed=M + N + K)
+    C = lime.map_matmul_bf16(_bf(A), _bf(Bt)).cpu().numpy()
+    e, fro = _check(C, A, Bt)
+    assert e <= MATMUL_RTOL and fro <= MATMUL_RTOL, (M, N, K, e, fro)
+
+
+def test_matmul_identity_exact(lime):
+    K = 256
+    A = inputs.bf16_uniform(300, K, 5, 0)
+    I = inputs._f32_to_bf16_bits(np.eye(K, dtype=np.float32))
+    C = lime.map_matmul_bf16(_bf(A), _bf(I)).cpu().numpy()
+    assert np.array_equal(C, inputs.bf16_bits_to_f32(A))
+
+
+def test_matmul_config4_sampled(lime):
+    M = N = K = 8192
+    A, Bt = inputs.matmul_operands(M, N, K, seed=4)
+    C = lime.map_matmul_bf16(_bf(A), _bf(Bt)).cpu().numpy()
+    rng = np.random.default_rng(1)
+    r = rng.integers(0, M, 65536)
+    c = rng.integers(0, N, 65536)
+    e, _ = _check(C, A, Bt, r, c)
+    assert e <= MATMUL_RTOL, e
+    rows = rng.integers(0, M, 16)
+    for i in rows:
+        e, _ = _check(C, A, Bt, np.full(N, i), np.arange(N))
+        assert e <= MATMUL_RTOL, (i, e)
+    cols = rng.integers(0, N, 16)
+    for j in cols:
+        e, _ = _check(C, A, Bt, np.arange(M), np.full(M, j))
+        assert e <= MATMUL_RTOL, (j, e)
+
+
+def test_matmul_launch_independent(lime):
+    A, Bt = inputs.matmul_operands(1024, 1024, 512, seed=9)
+    C0 = lime.map_matmul_bf16(_bf(A), _bf(Bt))
+    for g in (1, 7, 64):
+        with lime.launch_override(grid_ctas=g):
+            assert torch.equal(lime.map_matmul_bf16(_bf(A), _bf(Bt)), C0)

@@ -1,0 +1,60 @@
+"""SASS-level guards (no GPU): the compiled liblime.so must contain the instructions the design
+relies on. cuobjdump runs on the CPU box."""
+import re
+import shutil
+import subprocess
+
+import pytest
+
+from paper_conf_pldi_dubachcrbf12_b200 import build as lime_build
+
+pytestmark = pytest.mark.skipif(shutil.which("cuobjdump") is None, reason="cuobjdump not available")
+
+
+@pytest.fixture(scope="module")
+def sass():
+    lib = lime_build.build()
+    out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True, check=True).stdout
+    funcs, cur = {}, None
+    for line in out.splitlines():
+        m = re.search(r"Function : (\S+)", line)
+        if m:
+            cur = m.group(1)
+            funcs[cur] = []
+        elif cur and re.match(r"\s+/\*[0-9a-f]{4}\*/", line):
+            funcs[cur].append(re.sub(r"^\s+/\*[0-9a-f]+\*/\s+", "", line).split(";")[0])
+    return funcs
+
+
+def _fn(sass, pat):
+    hits = [k for k in sass if re.search(pat, k)]
+    assert hits, pat
+    return [i for k in hits for i in sass[k]]
+
+
+def test_mandelbrot_has_no_inexact_fma(sass):
+    # R7 bit-exactness: every FFMA/FFMA2 in the Mandelbrot kernel must be an exact rewrite of a
+    # single op (multiplier +-1 immediate), never a contracted x*y+z.
+    for ins in _fn(sass, r"mandel"):
+        if re.match(r"(@!?P\d )?FFMA", ins):
+            assert re.search(r",\s*-?1(\.0+)?\s*,", ins), ins
+
+
+def test_mandelbrot_uses_packed_fp32(sass):
+    ops = " ".join(_fn(sass, r"mandel"))
+    assert "FMUL2" in ops and "FADD2" in ops
+
+
+def test_nbody_uses_packed_fp32_and_mufu_and_bulk_copy(sass):
+    ops = " ".join(_fn(sass, r"force_kernelILi256ELi4ELb1"))
+    assert "FFMA2" in ops and "MUFU.RSQ" in ops
+    assert "UBLKCP" in ops                         # cp.async.bulk (1-D TMA) staging of j-tiles
+    assert "LDS.128" in ops                        # broadcast reads of the staged sources
+
+
+def test_gemm_is_tcgen05(sass):
+    ops = " ".join(_fn(sass, r"gemm_kernel"))
+    assert "UTCHMMA" in ops or "UTCQMMA" in ops   # tcgen05.mma
+    assert "UTMALDG" in ops                        # TMA tensor loads
+    assert "LDTM" in ops                           # tcgen05.ld epilogue
+    assert "HMMA" not in ops.replace("UTCHMMA", "")
