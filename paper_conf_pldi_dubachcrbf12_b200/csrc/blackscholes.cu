@@ -6,8 +6,9 @@
 // variant never writes call/put; fp64 partials per thread -> warp shuffle -> CTA ->
 // last CTA combines CTA partials in index order.
 //
-// The element function is written for B200's ridge point: 7 MUFU and ~45
-// FP32 lane-ops per option. Savings vs the textbook evaluation:
+// The element function is written for B200's ridge point: 6 MUFU and ~48
+// FP32 lane-ops per option, two options per packed FFMA2/FMUL2 instruction. Savings vs the
+// textbook evaluation:
 //   * 1/(sigma sqrt T) = rsqrt(T) / sigma  (one MUFU.RSQ gives both sqrt T and its inverse)
 //   * ln(S/X) = (lg2 S - lg2 X) ln 2
 //   * K phi(d2) = S phi(d1) (exact identity, K = X e^{-rT}) -> one exponential serves both
@@ -39,44 +40,89 @@ __device__ __forceinline__ float as_poly(float k) {
     return k * fmaf(k, fmaf(k, fmaf(k, fmaf(k, kAS_a5, kAS_a4), kAS_a3), kAS_a2), kAS_a1);
 }
 
-__device__ __forceinline__ void price(float S, float X, float T, const Consts& c, float& call, float& put) {
-    const float rsT = rsqrt_approx(T);
-    const float sqT = T * rsT;
-    const float v = c.sigma * sqT;                                   // sigma sqrt T
-    const float inv_v = rsT * c.inv_sigma;                           // 1 / (sigma sqrt T)
-    const float l = (lg2_approx(S) - lg2_approx(X)) * kLn2;         // ln(S/X)
-    const float d1 = fmaf(c.r_plus_half_s2, T, l) * inv_v;
-    const float d2 = d1 - v;
-    const float K = X * ex2_approx(c.neg_r_log2e * T);              // X e^{-rT}
-    const float k1 = rcp_approx(fmaf(kAS_p, fabsf(d1), 1.f));
-    const float k2 = rcp_approx(fmaf(kAS_p, fabsf(d2), 1.f));
-    const float sphi = S * (kInvSqrt2Pi * ex2_approx(kNegHalfLog2e * d1 * d1));   // S phi(d1) = K phi(d2)
-    const float sq1 = sphi * as_poly(k1);                           // S N(-|d1|)
-    const float kq2 = sphi * as_poly(k2);                           // K N(-|d2|)
-    const float sn1 = d1 >= 0.f ? S - sq1 : sq1;                    // S N(d1)
-    const float snm1 = d1 >= 0.f ? sq1 : S - sq1;                   // S N(-d1)
-    const float kn2 = d2 >= 0.f ? K - kq2 : kq2;                    // K N(d2)
-    const float knm2 = d2 >= 0.f ? kq2 : K - kq2;                   // K N(-d2)
-    call = sn1 - kn2;
-    put = knm2 - snm1;
+// Two options per call, packed (FFMA2/FMUL2/FADD2 carry both; MUFU ops are per lane).
+// Per option: 6 MUFU (rsqrt T, lg2 S, lg2 X, ex2 -rT, ex2 -d1^2/2, and ONE rcp shared by the two
+// Abramowitz-Stegun k's: k1 = D2/(D1 D2), k2 = D1/(D1 D2)).
+struct P2 { float2 call, put; };
+
+__device__ __forceinline__ float2 as_poly2(float2 k) {
+    float2 p = fma2(k, bcast2(kAS_a5), bcast2(kAS_a4));
+    p = fma2(k, p, bcast2(kAS_a3));
+    p = fma2(k, p, bcast2(kAS_a2));
+    p = fma2(k, p, bcast2(kAS_a1));
+    return mul2(k, p);
+}
+__device__ __forceinline__ float2 abs2(float2 v) { return make_float2(fabsf(v.x), fabsf(v.y)); }
+
+__device__ __forceinline__ P2 price2(float2 S, float2 X, float2 T, const Consts& c) {
+    const float2 rsT = make_float2(rsqrt_approx(T.x), rsqrt_approx(T.y));
+    const float2 sqT = mul2(T, rsT);
+    const float2 v = mul2(bcast2(c.sigma), sqT);                       // sigma sqrt T
+    const float2 inv_v = mul2(rsT, bcast2(c.inv_sigma));               // 1 / (sigma sqrt T)
+    const float2 lg = sub2(make_float2(lg2_approx(S.x), lg2_approx(S.y)),
+                           make_float2(lg2_approx(X.x), lg2_approx(X.y)));
+    const float2 l = mul2(lg, bcast2(kLn2));                            // ln(S/X)
+    const float2 d1 = mul2(fma2(bcast2(c.r_plus_half_s2), T, l), inv_v);
+    const float2 d2 = sub2(d1, v);
+    const float2 er = mul2(bcast2(c.neg_r_log2e), T);
+    const float2 K = mul2(X, make_float2(ex2_approx(er.x), ex2_approx(er.y)));   // X e^{-rT}
+    const float2 D1 = fma2(bcast2(kAS_p), abs2(d1), bcast2(1.f));
+    const float2 D2 = fma2(bcast2(kAS_p), abs2(d2), bcast2(1.f));
+    const float2 DD = mul2(D1, D2);
+    const float2 rr = make_float2(rcp_approx(DD.x), rcp_approx(DD.y));
+    const float2 k1 = mul2(D2, rr);                                     // 1 / D1
+    const float2 k2 = mul2(D1, rr);                                     // 1 / D2
+    const float2 g = mul2(mul2(bcast2(kNegHalfLog2e), d1), d1);
+    const float2 sphi = mul2(S, mul2(bcast2(kInvSqrt2Pi), make_float2(ex2_approx(g.x), ex2_approx(g.y))));
+    const float2 sq1 = mul2(sphi, as_poly2(k1));                       // S N(-|d1|)
+    const float2 kq2 = mul2(sphi, as_poly2(k2));                       // K N(-|d2|) = S phi(d1) poly(k2)
+    const float2 s_m = sub2(S, sq1);                                    // S (1 - N(-|d1|))
+    const float2 k_m = sub2(K, kq2);
+    P2 r;
+    const float sn1x = d1.x >= 0.f ? s_m.x : sq1.x, sn1y = d1.y >= 0.f ? s_m.y : sq1.y;       // S N(d1)
+    const float snm1x = d1.x >= 0.f ? sq1.x : s_m.x, snm1y = d1.y >= 0.f ? sq1.y : s_m.y;     // S N(-d1)
+    const float kn2x = d2.x >= 0.f ? k_m.x : kq2.x, kn2y = d2.y >= 0.f ? k_m.y : kq2.y;       // K N(d2)
+    const float knm2x = d2.x >= 0.f ? kq2.x : k_m.x, knm2y = d2.y >= 0.f ? kq2.y : k_m.y;     // K N(-d2)
+    r.call = sub2(make_float2(sn1x, sn1y), make_float2(kn2x, kn2y));
+    r.put = sub2(make_float2(knm2x, knm2y), make_float2(snm1x, snm1y));
+    return r;
 }
 
-__global__ void __launch_bounds__(256) map_kernel(const float* __restrict__ S, const float* __restrict__ X,
+__device__ __forceinline__ void price(float S, float X, float T, const Consts& c, float& call, float& put) {
+    const P2 r = price2(bcast2(S), bcast2(X), bcast2(T), c);
+    call = r.call.x;
+    put = r.put.x;
+}
+
+__device__ __forceinline__ void price4(const float4& s, const float4& x, const float4& t, const Consts& c,
+                                       float4& cv, float4& pv) {
+    const P2 a = price2(make_float2(s.x, s.y), make_float2(x.x, x.y), make_float2(t.x, t.y), c);
+    const P2 b = price2(make_float2(s.z, s.w), make_float2(x.z, x.w), make_float2(t.z, t.w), c);
+    cv = make_float4(a.call.x, a.call.y, b.call.x, b.call.y);
+    pv = make_float4(a.put.x, a.put.y, b.put.x, b.put.y);
+}
+
+__global__ void __launch_bounds__(256, 4) map_kernel(const float* __restrict__ S, const float* __restrict__ X,
                                                   const float* __restrict__ T, int64_t n, Consts c,
                                                   float* __restrict__ call, float* __restrict__ put) {
     const int64_t n4 = n >> 2;
     const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
-    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n4; i += stride) {
-        const float4 s = ld_stream_f4(reinterpret_cast<const float4*>(S) + i);
-        const float4 x = ld_stream_f4(reinterpret_cast<const float4*>(X) + i);
-        const float4 t = ld_stream_f4(reinterpret_cast<const float4*>(T) + i);
+    const float4* S4 = reinterpret_cast<const float4*>(S);
+    const float4* X4 = reinterpret_cast<const float4*>(X);
+    const float4* T4 = reinterpret_cast<const float4*>(T);
+    int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
+    float4 s, x, t;
+    if (i < n4) { s = ld_stream_f4(S4 + i); x = ld_stream_f4(X4 + i); t = ld_stream_f4(T4 + i); }
+    for (; i < n4; i += stride) {
+        // software pipeline: issue the next iteration's 48 B of loads before pricing this one
+        const int64_t nx = i + stride;
+        float4 s2 = s, x2 = x, t2 = t;
+        if (nx < n4) { s2 = ld_stream_f4(S4 + nx); x2 = ld_stream_f4(X4 + nx); t2 = ld_stream_f4(T4 + nx); }
         float4 cv, pv;
-        price(s.x, x.x, t.x, c, cv.x, pv.x);
-        price(s.y, x.y, t.y, c, cv.y, pv.y);
-        price(s.z, x.z, t.z, c, cv.z, pv.z);
-        price(s.w, x.w, t.w, c, cv.w, pv.w);
+        price4(s, x, t, c, cv, pv);
         st_stream_f4(reinterpret_cast<float4*>(call) + i, cv);
         st_stream_f4(reinterpret_cast<float4*>(put) + i, pv);
+        s = s2; x = x2; t = t2;
     }
     // ragged tail (n % 4 elements)
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (n & 3)) {
@@ -95,27 +141,33 @@ __device__ __forceinline__ double warp_sum(double v) {
 }
 
 // ws layout: [0]: u32 ticket counter; [256 B ...]: double2 CTA partials.
-__global__ void __launch_bounds__(256) map_reduce_kernel(const float* __restrict__ S, const float* __restrict__ X,
+__global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restrict__ S, const float* __restrict__ X,
                                                          const float* __restrict__ T, int64_t n, Consts c,
                                                          double* __restrict__ sums, unsigned* ticket,
                                                          double2* __restrict__ partial) {
     __shared__ double2 s_part[8];
     __shared__ int s_last;
-    double ac = 0.0, ap = 0.0;
+    // per-thread partials in fp32 (a thread prices ~n/(grid*256) options), fp64 from the warp up
+    float fc = 0.f, fp = 0.f;
     const int64_t n4 = n >> 2;
     const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
-    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n4; i += stride) {
-        const float4 s = ld_stream_f4(reinterpret_cast<const float4*>(S) + i);
-        const float4 x = ld_stream_f4(reinterpret_cast<const float4*>(X) + i);
-        const float4 t = ld_stream_f4(reinterpret_cast<const float4*>(T) + i);
-        float c0, c1, c2, c3, p0, p1, p2, p3;
-        price(s.x, x.x, t.x, c, c0, p0);
-        price(s.y, x.y, t.y, c, c1, p1);
-        price(s.z, x.z, t.z, c, c2, p2);
-        price(s.w, x.w, t.w, c, c3, p3);
-        ac += static_cast<double>((c0 + c1) + (c2 + c3));
-        ap += static_cast<double>((p0 + p1) + (p2 + p3));
+    const float4* S4 = reinterpret_cast<const float4*>(S);
+    const float4* X4 = reinterpret_cast<const float4*>(X);
+    const float4* T4 = reinterpret_cast<const float4*>(T);
+    int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
+    float4 s, x, t;
+    if (i < n4) { s = ld_stream_f4(S4 + i); x = ld_stream_f4(X4 + i); t = ld_stream_f4(T4 + i); }
+    for (; i < n4; i += stride) {
+        const int64_t nx = i + stride;
+        float4 s2 = s, x2 = x, t2 = t;
+        if (nx < n4) { s2 = ld_stream_f4(S4 + nx); x2 = ld_stream_f4(X4 + nx); t2 = ld_stream_f4(T4 + nx); }
+        float4 cv, pv;
+        price4(s, x, t, c, cv, pv);
+        fc += (cv.x + cv.y) + (cv.z + cv.w);
+        fp += (pv.x + pv.y) + (pv.z + pv.w);
+        s = s2; x = x2; t = t2;
     }
+    double ac = fc, ap = fp;
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (n & 3)) {
         const int64_t e = (n4 << 2) + threadIdx.x;
         float cv, pv;

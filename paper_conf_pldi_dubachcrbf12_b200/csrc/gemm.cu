@@ -232,6 +232,216 @@ gemm_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ 
     }
 }
 
+// =====================================================================================
+// 2-CTA variant (cta_group::2): a CTA pair on one TPC computes a 256 x 256 tile. Each CTA stages
+// its 128-row half of A and its 128-row half of Bt (per K-slice: 16 + 16 KB), so each SM's smem
+// and L2 traffic per flop is 2/3 of the 1-CTA 128 x 256 tile's; the leader CTA's single thread
+// issues tcgen05.mma.cta_group::2 (M = 256, N = 256, K = 16) reading both CTAs' smem, and each
+// CTA's TMEM receives its own 128 accumulator rows.
+// =====================================================================================
+namespace two {
+constexpr int BM = 128;                 // rows of A per CTA (pair tile: 256)
+constexpr int BN = 256;                 // pair tile N (each CTA stages 128 rows of Bt)
+constexpr int STAGES = 6;
+constexpr uint32_t kStageA = BM * BK * 2;            // 16 KB
+constexpr uint32_t kStageB = (BN / 2) * BK * 2;      // 16 KB
+constexpr uint32_t kStageBytes = kStageA + kStageB;
+constexpr size_t kSmemBytes = 1024 + STAGES * kStageBytes + 256;
+constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(BN >> 3) << 17) |
+                            (static_cast<uint32_t>(256 >> 4) << 24);
+}  // namespace two
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t saddr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" :: "r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx_cluster(uint32_t cluster_addr, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.release.cluster.shared::cluster.b64 _, [%0], %1;"
+                 :: "r"(cluster_addr), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap* map, void* dst, uint32_t leader_bar, int c0, int c1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+        :: "r"(smem_addr(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(leader_bar)
+        : "memory");
+}
+__device__ __forceinline__ void tc_mma_pair(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc) : "memory");
+}
+__device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+                 :: "r"(smem_addr(bar)), "h"(static_cast<uint16_t>(3)) : "memory");
+}
+
+struct Params2 {
+    float* C;
+    int M, N, K;
+    int num_m, num_n, num_k;   // num_m counts 256-row pair tiles
+    int num_tiles;
+};
+
+__device__ __forceinline__ void tile_coords2(int t, const Params2& p, int& mb, int& nb) {
+    constexpr int G = 8;       // raster group of pair-tile rows sharing Bt tiles in L2
+    const int per_group = G * p.num_n;
+    const int g = t / per_group;
+    const int first_m = g * G;
+    const int gm = min(p.num_m - first_m, G);
+    const int r = t - g * per_group;
+    mb = first_m + r % gm;
+    nb = r / gm;
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+             const __grid_constant__ Params2 p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + two::STAGES * two::kStageBytes);
+    uint64_t* empty = full + two::STAGES;
+    uint64_t* tfull = empty + two::STAGES;
+    uint64_t* tempty = tfull + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+    const bool leader = (rank == 0);
+    const int cluster = blockIdx.x >> 1;
+    const int nclusters = gridDim.x >> 1;
+
+    if (warp == 0 && lane == 0) {
+        prefetch_tmap(&tmap_a);
+        prefetch_tmap(&tmap_b);
+        for (int s = 0; s < two::STAGES; ++s) {
+            mbar_init(&full[s], 1);      // leader's producer arms it with both CTAs' tx bytes
+            mbar_init(&empty[s], 1);     // released by the leader's MMA commit (multicast to both CTAs)
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull[a], 1);
+            mbar_init(&tempty[a], 8);    // 4 epilogue warps x 2 CTAs (leader's copy is the one used)
+        }
+        fence_mbar_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_addr(tmem_slot)), "r"(kTmemCols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
+    tc_fence_before();
+    cluster_sync();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int t = cluster; t < p.num_tiles; t += nclusters) {
+                int mb, nb;
+                tile_coords2(t, p, mb, nb);
+                const int arow = mb * 256 + static_cast<int>(rank) * two::BM;
+                const int brow = nb * two::BN + static_cast<int>(rank) * (two::BN / 2);
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&empty[s], ph ^ 1);
+                    uint8_t* sa = smem + s * two::kStageBytes;
+                    const uint32_t lbar = mapa_shared(smem_addr(&full[s]), 0);
+                    // only the leader arms its barrier, for both CTAs' bytes; the peer's TMA
+                    // complete_tx lands on the same barrier (no remote arrive on the hot loop)
+                    if (leader) mbar_arrive_expect_tx(&full[s], 2 * two::kStageBytes);
+                    tma_load_2d_pair(&tmap_a, sa, lbar, kb * BK, arow);
+                    tma_load_2d_pair(&tmap_b, sa + two::kStageA, lbar, kb * BK, brow);
+                    if (++s == two::STAGES) { s = 0; ph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (leader && lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            int local = 0;
+            for (int t = cluster; t < p.num_tiles; t += nclusters, ++local) {
+                const int acc = local & 1;
+                mbar_wait(&tempty[acc], ((local >> 1) & 1) ^ 1);
+                tc_fence_after();
+                const uint32_t dtm = tmem_base + static_cast<uint32_t>(acc * two::BN);
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&full[s], ph);
+                    tc_fence_after();
+                    const uint32_t sa = smem_addr(smem + s * two::kStageBytes);
+                    const uint32_t sb = sa + two::kStageA;
+#pragma unroll
+                    for (int k = 0; k < BK / UMMA_K; ++k)
+                        tc_mma_pair(dtm, smem_desc_sw128(sa + k * UMMA_K * 2), smem_desc_sw128(sb + k * UMMA_K * 2),
+                                    two::kIdesc, (kb | k) != 0);
+                    tc_commit_pair(&empty[s]);
+                    if (++s == two::STAGES) { s = 0; ph ^= 1; }
+                }
+                tc_commit_pair(&tfull[acc]);
+            }
+        }
+        __syncwarp();
+    } else {
+        const int quad = warp & 3;
+        const int row_in_tile = quad * 32 + lane;
+        const uint32_t tempty_leader0 = mapa_shared(smem_addr(&tempty[0]), 0);
+        int local = 0;
+        for (int t = cluster; t < p.num_tiles; t += nclusters, ++local) {
+            const int acc = local & 1;
+            int mb, nb;
+            tile_coords2(t, p, mb, nb);
+            mbar_wait(&tfull[acc], (local >> 1) & 1);
+            tc_fence_after();
+            const int row = mb * 256 + static_cast<int>(rank) * two::BM + row_in_tile;
+            const uint32_t tbase = tmem_base + (static_cast<uint32_t>(quad * 32) << 16) + static_cast<uint32_t>(acc * two::BN);
+            float* crow = p.C + static_cast<int64_t>(row) * p.N;
+            const bool vec_ok = (p.N & 3) == 0;
+#pragma unroll 1
+            for (int c = 0; c < two::BN; c += 32) {
+                float v[32];
+                tmem_ld32(tbase + c, v);
+                const int col0 = nb * two::BN + c;
+                if (row < p.M) {
+                    if (vec_ok && col0 + 32 <= p.N) {
+#pragma unroll
+                        for (int q = 0; q < 8; ++q)
+                            st_stream_f4(reinterpret_cast<float4*>(crow + col0) + q,
+                                         make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]));
+                    } else {
+#pragma unroll
+                        for (int q = 0; q < 32; ++q)
+                            if (col0 + q < p.N) crow[col0 + q] = v[q];
+                    }
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cluster(tempty_leader0 + static_cast<uint32_t>(acc * 8));
+        }
+    }
+
+    tc_fence_before();
+    cluster_sync();
+    if (warp == 1) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(tmem_base), "r"(kTmemCols) : "memory");
+    }
+}
+
 // ------------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -259,7 +469,32 @@ static bool make_map(CUtensorMap* map, const void* base, uint64_t rows, uint64_t
 
 cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
                         cudaStream_t stream) {
+    const LaunchOverride& ov = launch_override();
+    const bool pair = ov.per_thread == 2 || (ov.per_thread != 1 && M >= 256);
     CUtensorMap ma, mb;
+    if (pair) {
+        if (!make_map(&ma, A, M, K, two::BM) || !make_map(&mb, Bt, N, K, two::BN / 2)) return cudaErrorInvalidValue;
+        Params2 p;
+        p.C = C;
+        p.M = static_cast<int>(M);
+        p.N = static_cast<int>(N);
+        p.K = static_cast<int>(K);
+        p.num_m = static_cast<int>(ceil_div<int64_t>(M, 256));
+        p.num_n = static_cast<int>(ceil_div<int64_t>(N, two::BN));
+        p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
+        p.num_tiles = p.num_m * p.num_n;
+        static bool attr2 = false;
+        if (!attr2) {
+            cudaError_t e = cudaFuncSetAttribute(gemm2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                 static_cast<int>(two::kSmemBytes));
+            if (e != cudaSuccess) return e;
+            attr2 = true;
+        }
+        int clusters = ov.grid_ctas > 0 ? mx(1, ov.grid_ctas / 2) : device_num_sms() / 2;
+        clusters = mn(clusters, p.num_tiles);
+        gemm2_kernel<<<2 * clusters, kThreads, two::kSmemBytes, stream>>>(ma, mb, p);
+        return cudaGetLastError();
+    }
     if (!make_map(&ma, A, M, K, BM) || !make_map(&mb, Bt, N, K, BN)) return cudaErrorInvalidValue;
     Params p;
     p.C = C;
@@ -277,7 +512,7 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    int grid = launch_override().grid_ctas;
+    int grid = ov.grid_ctas;
     if (grid <= 0) grid = device_num_sms();
     grid = mn(grid, p.num_tiles);
     gemm_kernel<<<grid, kThreads, kSmemBytes, stream>>>(ma, mb, p);

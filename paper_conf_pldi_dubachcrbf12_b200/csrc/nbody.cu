@@ -125,20 +125,36 @@ struct Interact<R, true> {
 #pragma unroll
         for (int q = 0; q < Q; ++q) { ax[q] = add2(ax[q], cx[q]); ay[q] = add2(ay[q], cy[q]); az[q] = add2(az[q], cz[q]); }
     }
+    // Stage-interleaved across the Q target pairs (each stage is Q independent packed ops), so a
+    // warp always has Q-wide ILP between dependent steps; per-lane op order equals the scalar path.
     __device__ __forceinline__ void body(const float4 b, const float eps2) {
         const float2 e2 = bcast2(eps2);
+        float2 dx[Q], dy[Q], dz[Q], r2[Q], inv[Q], t[Q];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dz[q] = sub2(bcast2(b.z), pz[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dz[q], dz[q], e2);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dy[q] = sub2(bcast2(b.y), py[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dy[q], dy[q], r2[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dx[q] = sub2(bcast2(b.x), px[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dx[q], dx[q], r2[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) inv[q] = make_float2(rsqrt_approx(r2[q].x), rsqrt_approx(r2[q].y));
+#pragma unroll
+        for (int q = 0; q < Q; ++q) t[q] = mul2(bcast2(b.w), inv[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) inv[q] = mul2(inv[q], inv[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) t[q] = mul2(t[q], inv[q]);            // s = (m_j inv) inv^2
 #pragma unroll
         for (int q = 0; q < Q; ++q) {
-            const float2 dx = sub2(bcast2(b.x), px[q]);
-            const float2 dy = sub2(bcast2(b.y), py[q]);
-            const float2 dz = sub2(bcast2(b.z), pz[q]);
-            const float2 r2 = fma2(dx, dx, fma2(dy, dy, fma2(dz, dz, e2)));
-            const float2 inv = make_float2(rsqrt_approx(r2.x), rsqrt_approx(r2.y));
-            const float2 inv2 = mul2(inv, inv);
-            const float2 s = mul2(mul2(bcast2(b.w), inv), inv2);
-            cx[q] = fma2(s, dx, cx[q]);
-            cy[q] = fma2(s, dy, cy[q]);
-            cz[q] = fma2(s, dz, cz[q]);
+            cx[q] = fma2(t[q], dx[q], cx[q]);
+            cy[q] = fma2(t[q], dy[q], cy[q]);
+            cz[q] = fma2(t[q], dz[q], cz[q]);
         }
     }
     __device__ __forceinline__ float4 result(int r) const {
@@ -276,11 +292,13 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     const LaunchOverride& ov = launch_override();
     int block = ov.block_threads, R = ov.per_thread;
     if (block == 0 || R == 0) {
-        // Automatic: the largest target tile that still gives >= 4 CTAs per SM of work items.
-        const int64_t want = 4LL * device_num_sms();
-        const int cand[][2] = {{256, 4}, {256, 2}, {128, 2}, {128, 1}};
-        int pick = 3;
-        for (int k = 0; k < 4; ++k) {
+        // Automatic (tools/tune_nbody.py sweep on B200, profiles/tune_nbody_r01.jsonl): 256 threads x
+        // 2 targets (one packed pair) is fastest at 2^20; small problems drop to 128-thread tiles so
+        // that there are >= 1.5 work items per SM.
+        const int64_t want = 3LL * device_num_sms() / 2;
+        const int cand[][2] = {{256, 2}, {128, 2}, {128, 1}};
+        int pick = 2;
+        for (int k = 0; k < 3; ++k) {
             const int64_t items = ceil_div<int64_t>(tgt_count, cand[k][0] * cand[k][1]) * a.splits;
             if (items >= want) { pick = k; break; }
         }
