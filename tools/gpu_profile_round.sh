@@ -10,7 +10,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
     python bench.py --steps 3 --warmup 3 > gpurun_out/bench_under_ncu_${TAG}.json 2>&1
 echo "launch list rc=$?"
 declare -A KRE=( [nbody1m]=force_kernel [nbody1m_p8]=force_kernel [nbody4096]=force_kernel [bs_map]=map_kernel
-                 [bs_fused]=map_reduce_kernel [mandel]=mandel_kernel [matmul]=gemm_kernel [reduce]=reduce_kernel )
+                 [bs_fused]=map_reduce_kernel [mandel]=mandel_kernel [matmul]=gemm [reduce]=reduce_kernel )
 for k in $KERNELS; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:${KRE[$k]} -s 1 -c 1 \
       -o gpurun_out/prof_${k}_${TAG} -f python tools/prof_kernels.py $k 2 > gpurun_out/prof_${k}_${TAG}.log 2>&1

@@ -97,6 +97,65 @@ __global__ void k_ex2(float* out, float a, float b, int iters) {
     if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
 }
 
+__global__ void k_dfma(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    double x[CH];
+    const double A = a, B = b;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = threadIdx.x * 1e-3 + c;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = fma(x[c], A, B);
+    double s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.0) out[0] = (float)s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+
+// 8 FFMA2 chains + 4 DFMA chains per iteration: if the FP64 pipe runs beside the FP32 pipe, time
+// stays at the FFMA2-only time (lane_ops counted = FP32 lanes only).
+__global__ void k_mix(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float2 x[CH];
+    double y[4];
+    const float2 A = make_float2(a, a), B = make_float2(b, b);
+    const double Ad = a, Bd = b;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = make_float2(threadIdx.x * 1e-3f + c, c);
+#pragma unroll
+    for (int c = 0; c < 4; ++c) y[c] = threadIdx.x * 1e-3 + c;
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = ffma2(x[c], A, B);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) y[c] = fma(y[c], Ad, Bd);
+    }
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c].x + x[c].y;
+    for (int c = 0; c < 4; ++c) s += (float)y[c];
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+
+// F2F.F64.F32 conversion rate
+__global__ void k_f2d(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float x[CH];
+    double acc = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = threadIdx.x * 1e-3f + c;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) { x[c] = (float)((double)x[c] * 0.999); }
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.f) out[0] = s + (float)acc;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+
 __global__ void k_read(const float4* __restrict__ in, size_t n4, float* out) {
     float4 acc = make_float4(0, 0, 0, 0);
     for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n4; i += (size_t)gridDim.x * blockDim.x) {
@@ -147,6 +206,8 @@ int main() {
     struct { const char* name; void (*k)(float*, float, float, int); double lane_ops_per_iter; } tests[] = {
         {"ffma", k_ffma, CH}, {"ffma2", k_ffma2, 2.0 * CH}, {"fadd2", k_fadd2, 2.0 * CH},
         {"mufu_rsq", k_rsq, CH}, {"mufu_ex2(+fmul)", k_ex2, CH},
+        {"dfma(fp64 lanes)", k_dfma, CH}, {"ffma2+dfma(fp32 lanes only)", k_mix, 2.0 * CH},
+        {"f32->f64->f32 roundtrips(+dmul)", k_f2d, CH},
     };
     for (auto& t : tests) {
         float ms = time_it([&] { t.k<<<blocks, threads>>>(out, 0.999f, 1e-3f, iters); }, 5);

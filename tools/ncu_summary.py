@@ -24,6 +24,7 @@ KEYS = {
     "launch__grid_size": "grid",
     "launch__block_size": "block",
     "sm__cycles_elapsed.avg.per_second": "sm_hz",
+    "lts__throughput.avg.pct_of_peak_sustained_elapsed": "l2_throughput_pct",
     "lts__t_bytes.sum": "l2_bytes",
     "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum": "smem_ld_bank_conflicts",
     "smsp__thread_inst_executed_per_inst_executed.ratio": "threads_per_inst",
@@ -48,11 +49,11 @@ def summarize(rep):
                 except ValueError:
                     pass
                 u = units[hdr.index(k)]
-                if u == "Kbyte" and isinstance(v, float): v *= 1e3
-                if u == "Mbyte" and isinstance(v, float): v *= 1e6
-                if u == "Gbyte" and isinstance(v, float): v *= 1e9
-                if u == "usecond" and isinstance(v, float): v *= 1e3
-                if u == "msecond" and isinstance(v, float): v *= 1e6
+                scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+                         "ns": 1, "nsecond": 1, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6,
+                         "s": 1e9, "second": 1e9, "Ghz": 1e9, "Mhz": 1e6, "hz": 1}.get(u)
+                if scale is not None and isinstance(v, float):
+                    v *= scale
                 d[nm] = v
         # stall reasons
         stalls = {}
