@@ -97,6 +97,37 @@ __global__ void k_ex2(float* out, float a, float b, int iters) {
     if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
 }
 
+__device__ __forceinline__ float lg2f(float x) { float y; asm volatile("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
+__device__ __forceinline__ float rcpf(float x) { float y; asm volatile("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
+__global__ void k_lg2(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = 3.0f + threadIdx.x * 1e-3f + c;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = lg2f(x[c]) + 2.5f;
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+__global__ void k_rcp(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = 1.5f + threadIdx.x * 1e-3f + c;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = rcpf(x[c]);
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+
 __global__ void k_dfma(float* out, float a, float b, int iters) {
     long long t0 = clock64();
     double x[CH];
@@ -206,6 +237,7 @@ int main() {
     struct { const char* name; void (*k)(float*, float, float, int); double lane_ops_per_iter; } tests[] = {
         {"ffma", k_ffma, CH}, {"ffma2", k_ffma2, 2.0 * CH}, {"fadd2", k_fadd2, 2.0 * CH},
         {"mufu_rsq", k_rsq, CH}, {"mufu_ex2(+fmul)", k_ex2, CH},
+        {"mufu_lg2(+fadd)", k_lg2, CH}, {"mufu_rcp", k_rcp, CH},
         {"dfma(fp64 lanes)", k_dfma, CH}, {"ffma2+dfma(fp32 lanes only)", k_mix, 2.0 * CH},
         {"f32->f64->f32 roundtrips(+dmul)", k_f2d, CH},
     };
