@@ -208,241 +208,6 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
     }
 }
 
-// ---------------------------------------------------------------------------------------------
-// Per-warp TMA pipelines (default variant). Each warp streams its own sequence of 128-option warp
-// tiles (32 lanes x one float4 of S, X and T = 3 x 512 B) through a kWStages-deep ring of
-// warp-private shared-memory slots: lane 0 issues the three 1-D bulk copies (cp.async.bulk +
-// mbarrier complete_tx) kWStages-1 tiles ahead, lanes read their float4s back with LDS.128. No
-// block-wide barrier, so warps never wait for each other, and the bytes in flight (up to
-// 3 tiles x 1.5 KB per warp, 32 warps per SM) do not cost registers.
-// ---------------------------------------------------------------------------------------------
-constexpr int kWThreads = 128;
-constexpr int kWStages = 4;
-constexpr uint32_t kWTileBytes = 32 * 16;     // per operand per warp tile
-
-struct WArgs {
-    const float* S;
-    const float* X;
-    const float* T;
-    int64_t n;
-    Consts c;
-    float* call;
-    float* put;
-    double* sums;
-    unsigned* ticket;
-    double2* partial;
-};
-
-template <bool kFused>
-__global__ void __launch_bounds__(kWThreads, 8) bs_warp_kernel(const __grid_constant__ WArgs a) {
-    constexpr int kWarps = kWThreads / 32;
-    __shared__ __align__(128) float4 ring[kWarps][kWStages][3][32];
-    __shared__ __align__(8) uint64_t full[kWarps][kWStages];
-    __shared__ double2 s_part[kWarps];
-    __shared__ int s_last;
-
-    const int warp = threadIdx.x >> 5;
-    const unsigned lane = lane_id();
-    const int64_t n4 = a.n >> 2;
-    const int64_t wtiles = ceil_div<int64_t>(n4, 32);
-    const int64_t gw = static_cast<int64_t>(blockIdx.x) * kWarps + warp;
-    const int64_t nw = static_cast<int64_t>(gridDim.x) * kWarps;
-    const int64_t my = gw < wtiles ? ceil_div<int64_t>(wtiles - gw, nw) : 0;
-
-    if (lane == 0) {
-        for (int st = 0; st < kWStages; ++st) mbar_init(&full[warp][st], 1);
-        fence_mbar_init();
-    }
-    __syncwarp();
-    auto issue = [&](int64_t k) {
-        const int64_t g0 = (gw + k * nw) * 32;
-        const uint32_t bytes = static_cast<uint32_t>(mn<int64_t>(32, n4 - g0)) * 16u;
-        const int st = static_cast<int>(k % kWStages);
-        mbar_arrive_expect_tx(&full[warp][st], 3 * bytes);
-        bulk_g2s(ring[warp][st][0], a.S + 4 * g0, bytes, &full[warp][st]);
-        bulk_g2s(ring[warp][st][1], a.X + 4 * g0, bytes, &full[warp][st]);
-        bulk_g2s(ring[warp][st][2], a.T + 4 * g0, bytes, &full[warp][st]);
-    };
-    if (lane == 0)
-        for (int64_t k = 0; k < mn<int64_t>(kWStages - 1, my); ++k) issue(k);
-
-    float fc = 0.f, fp = 0.f;
-    for (int64_t k = 0; k < my; ++k) {
-        if (lane == 0 && k + kWStages - 1 < my) issue(k + kWStages - 1);   // slot (k-1) % kWStages
-        const int st = static_cast<int>(k % kWStages);
-        mbar_wait(&full[warp][st], static_cast<uint32_t>((k / kWStages) & 1));
-        const int64_t g = (gw + k * nw) * 32 + lane;
-        if (g < n4) {
-            const float4 s = ring[warp][st][0][lane];
-            const float4 x = ring[warp][st][1][lane];
-            const float4 t = ring[warp][st][2][lane];
-            float4 cv, pv;
-            price4(s, x, t, a.c, cv, pv);
-            if (kFused) {
-                fc += (cv.x + cv.y) + (cv.z + cv.w);
-                fp += (pv.x + pv.y) + (pv.z + pv.w);
-            } else {
-                st_stream_f4(reinterpret_cast<float4*>(a.call) + g, cv);
-                st_stream_f4(reinterpret_cast<float4*>(a.put) + g, pv);
-            }
-        }
-        __syncwarp();                                                        // slot st read by all lanes
-    }
-    double ac = fc, ap = fp;
-    if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (a.n & 3)) {        // ragged tail (n % 4)
-        const int64_t e = (n4 << 2) + threadIdx.x;
-        float cv, pv;
-        price(a.S[e], a.X[e], a.T[e], a.c, cv, pv);
-        if (kFused) {
-            ac += cv;
-            ap += pv;
-        } else {
-            a.call[e] = cv;
-            a.put[e] = pv;
-        }
-    }
-    if (!kFused) return;
-
-    ac = warp_sum(ac);
-    ap = warp_sum(ap);
-    if (lane == 0) s_part[warp] = make_double2(ac, ap);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        double2 b = s_part[0];
-        for (int w = 1; w < kWarps; ++w) { b.x += s_part[w].x; b.y += s_part[w].y; }
-        __stcg(a.partial + blockIdx.x, b);
-        __threadfence();
-        s_last = (atomicAdd(a.ticket, 1u) == gridDim.x - 1);
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    if (warp == 0) {
-        double bx = 0.0, by = 0.0;
-        for (unsigned k = lane; k < gridDim.x; k += 32) {
-            const double2 pp = __ldcg(a.partial + k);
-            bx += pp.x;
-            by += pp.y;
-        }
-        bx = warp_sum(bx);
-        by = warp_sum(by);
-        if (lane == 0) {
-            a.sums[0] = bx;
-            a.sums[1] = by;
-            *a.ticket = 0u;
-        }
-    }
-}
-
-template <bool kFused>
-static int wgrid_for(int64_t n) {
-    const int ov = launch_override().grid_ctas;
-    if (ov > 0) return ov;
-    static int per_sm = 0;
-    if (per_sm == 0) {
-        int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bs_warp_kernel<kFused>, kWThreads, 0);
-        per_sm = b > 0 ? b : 1;
-    }
-    const int64_t need = mx<int64_t>(1, ceil_div<int64_t>(n >> 2, kWThreads));
-    return static_cast<int>(mn<int64_t>(need, static_cast<int64_t>(per_sm) * device_num_sms()));
-}
-
-// ---------------------------------------------------------------------------------------------
-// Light variant: one packed pair of options per thread-iteration (LDG.64 of each operand, a
-// two-deep register prefetch), so the per-thread footprint stays small and 48 warps per SM can be
-// resident to hide HBM latency behind the MUFU/FMA work.
-// ---------------------------------------------------------------------------------------------
-template <bool kFused>
-__global__ void __launch_bounds__(256, 6) bs_pair_kernel(const __grid_constant__ WArgs a) {
-    __shared__ double2 s_part[8];
-    __shared__ int s_last;
-    const int64_t n2 = a.n >> 1;
-    const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
-    const float2* S2 = reinterpret_cast<const float2*>(a.S);
-    const float2* X2 = reinterpret_cast<const float2*>(a.X);
-    const float2* T2 = reinterpret_cast<const float2*>(a.T);
-    auto ld2 = [](const float2* p) {
-        float2 v;
-        asm volatile("ld.global.nc.L1::no_allocate.v2.f32 {%0,%1}, [%2];" : "=f"(v.x), "=f"(v.y) : "l"(p));
-        return v;
-    };
-    int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
-    float2 s0 = make_float2(1.f, 1.f), x0 = s0, t0 = s0, s1 = s0, x1 = s0, t1 = s0;
-    if (i < n2) { s0 = ld2(S2 + i); x0 = ld2(X2 + i); t0 = ld2(T2 + i); }
-    if (i + stride < n2) { s1 = ld2(S2 + i + stride); x1 = ld2(X2 + i + stride); t1 = ld2(T2 + i + stride); }
-    float fc = 0.f, fp = 0.f;
-    for (; i < n2; i += stride) {
-        const int64_t nx = i + 2 * stride;
-        float2 s2 = s1, x2 = x1, t2 = t1;
-        if (nx < n2) { s2 = ld2(S2 + nx); x2 = ld2(X2 + nx); t2 = ld2(T2 + nx); }
-        const P2 r = price2(s0, x0, t0, a.c);
-        if (kFused) {
-            fc += r.call.x + r.call.y;
-            fp += r.put.x + r.put.y;
-        } else {
-            asm volatile("st.global.cs.v2.f32 [%0], {%1,%2};" :: "l"(reinterpret_cast<float2*>(a.call) + i),
-                         "f"(r.call.x), "f"(r.call.y) : "memory");
-            asm volatile("st.global.cs.v2.f32 [%0], {%1,%2};" :: "l"(reinterpret_cast<float2*>(a.put) + i),
-                         "f"(r.put.x), "f"(r.put.y) : "memory");
-        }
-        s0 = s1; x0 = x1; t0 = t1;
-        s1 = s2; x1 = x2; t1 = t2;
-    }
-    double ac = fc, ap = fp;
-    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0 && (a.n & 1)) {   // ragged tail
-        const int64_t e = a.n - 1;
-        float cv, pv;
-        price(a.S[e], a.X[e], a.T[e], a.c, cv, pv);
-        if (kFused) { ac += cv; ap += pv; } else { a.call[e] = cv; a.put[e] = pv; }
-    }
-    if (!kFused) return;
-    ac = warp_sum(ac);
-    ap = warp_sum(ap);
-    const int warp = threadIdx.x >> 5;
-    if (lane_id() == 0) s_part[warp] = make_double2(ac, ap);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        double2 b = s_part[0];
-        for (int w = 1; w < (blockDim.x >> 5); ++w) { b.x += s_part[w].x; b.y += s_part[w].y; }
-        __stcg(a.partial + blockIdx.x, b);
-        __threadfence();
-        s_last = (atomicAdd(a.ticket, 1u) == gridDim.x - 1);
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    if (warp == 0) {
-        double bx = 0.0, by = 0.0;
-        for (unsigned k = lane_id(); k < gridDim.x; k += 32) {
-            const double2 pp = __ldcg(a.partial + k);
-            bx += pp.x;
-            by += pp.y;
-        }
-        bx = warp_sum(bx);
-        by = warp_sum(by);
-        if (lane_id() == 0) {
-            a.sums[0] = bx;
-            a.sums[1] = by;
-            *a.ticket = 0u;
-        }
-    }
-}
-
-template <bool kFused>
-static int pgrid_for(int64_t n) {
-    const int ov = launch_override().grid_ctas;
-    if (ov > 0) return ov;
-    static int per_sm = 0;
-    if (per_sm == 0) {
-        int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, bs_pair_kernel<kFused>, 256, 0);
-        per_sm = b > 0 ? b : 1;
-    }
-    const int64_t need = mx<int64_t>(1, ceil_div<int64_t>(n >> 1, 256));
-    return static_cast<int>(mn<int64_t>(need, static_cast<int64_t>(per_sm) * device_num_sms()));
-}
-
 static Consts make_consts(float r, float sigma) {
     Consts c;
     c.r_plus_half_s2 = r + 0.5f * sigma * sigma;
@@ -466,46 +231,21 @@ static int grid_for(const void* kernel, int64_t n) {
     return static_cast<int>(mn<int64_t>(need, static_cast<int64_t>(per_sm[idx]) * device_num_sms()));
 }
 
-// launch override per_thread == 1 selects the register-prefetch variant (A/B comparisons)
 cudaError_t launch_map(const float* S, const float* X, const float* T, int64_t n, float r, float sigma,
                        float* call, float* put, cudaStream_t stream) {
     if (n == 0) return cudaSuccess;
-    if (launch_override().per_thread == 2) {
-        WArgs a{S, X, T, n, make_consts(r, sigma), call, put, nullptr, nullptr, nullptr};
-        bs_pair_kernel<false><<<pgrid_for<false>(n), 256, 0, stream>>>(a);
-        return cudaGetLastError();
-    }
-    if (launch_override().per_thread == 1) {
-        const int grid = grid_for(reinterpret_cast<const void*>(&map_kernel), n);
-        map_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), call, put);
-        return cudaGetLastError();
-    }
-    WArgs a{S, X, T, n, make_consts(r, sigma), call, put, nullptr, nullptr, nullptr};
-    bs_warp_kernel<false><<<wgrid_for<false>(n), kWThreads, 0, stream>>>(a);
+    const int grid = grid_for(reinterpret_cast<const void*>(&map_kernel), n);
+    map_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), call, put);
     return cudaGetLastError();
 }
 
 cudaError_t launch_map_reduce(const float* S, const float* X, const float* T, int64_t n, float r,
                               float sigma, double* sums, void* ws, cudaStream_t stream) {
+    int grid = grid_for(reinterpret_cast<const void*>(&map_reduce_kernel), n);
+    if (grid > red::kMaxCtas) grid = red::kMaxCtas;
     unsigned* ticket = static_cast<unsigned*>(ws);
     double2* partial = reinterpret_cast<double2*>(static_cast<char*>(ws) + 256);
-    if (launch_override().per_thread == 2) {
-        int grid = pgrid_for<true>(n);
-        if (grid > red::kMaxCtas) grid = red::kMaxCtas;
-        WArgs a{S, X, T, n, make_consts(r, sigma), nullptr, nullptr, sums, ticket, partial};
-        bs_pair_kernel<true><<<grid, 256, 0, stream>>>(a);
-        return cudaGetLastError();
-    }
-    if (launch_override().per_thread == 1) {
-        int grid = grid_for(reinterpret_cast<const void*>(&map_reduce_kernel), n);
-        if (grid > red::kMaxCtas) grid = red::kMaxCtas;
-        map_reduce_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), sums, ticket, partial);
-        return cudaGetLastError();
-    }
-    int grid = wgrid_for<true>(n);
-    if (grid > red::kMaxCtas) grid = red::kMaxCtas;
-    WArgs a{S, X, T, n, make_consts(r, sigma), nullptr, nullptr, sums, ticket, partial};
-    bs_warp_kernel<true><<<grid, kWThreads, 0, stream>>>(a);
+    map_reduce_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), sums, ticket, partial);
     return cudaGetLastError();
 }
 
