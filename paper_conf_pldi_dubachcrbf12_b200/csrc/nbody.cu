@@ -265,6 +265,82 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
     if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
 }
 
+// =====================================================================================
+// Small problems (n_src <= kSmallMaxSources, e.g. the paper's 4096 bodies, Table 3): the
+// splits live inside one CTA instead of across CTAs. A CTA owns 32 targets (one per lane) and has
+// one warp per split; warp w bulk-copies split w's sources (<= 8 KB) into its own smem slice and
+// runs exactly the arithmetic of the general kernel (scalar variant: chunk partials added into
+// the split accumulator in chunk order); the split partials are then added in split order from
+// shared memory. Same summation order as force_kernel, hence bit-identical results, but no global
+// partials, no atomic tickets and ~16 warps per SM instead of 1-2 CTAs of 4 warps.
+// =====================================================================================
+constexpr int64_t kSmallMaxSources = 8192;
+
+__global__ void __launch_bounds__(32 * kMaxSplits) force_small_kernel(const __grid_constant__ ForceArgs a) {
+    extern __shared__ __align__(128) uint8_t small_smem[];
+    float4* src = reinterpret_cast<float4*>(small_smem);                          // [S][split_len]
+    float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
+    __shared__ __align__(8) uint64_t bar[kMaxSplits];
+
+    const int warp = threadIdx.x >> 5;            // = split index
+    const unsigned lane = lane_id();
+    const int64_t t = static_cast<int64_t>(blockIdx.x) * 32 + lane;
+    const bool valid = t < a.tgt_count;
+    Interact<1, false> it;
+    it.set(0, __ldg(a.bodies + a.tgt_begin + (valid ? t : a.tgt_count - 1)));
+    it.zero_all();
+
+    const int64_t j0 = static_cast<int64_t>(warp) * a.split_len;
+    const int64_t j1 = mn<int64_t>(a.n_src, j0 + a.split_len);
+    const int len = static_cast<int>(j1 - j0);
+    float4* sb = src + static_cast<int64_t>(warp) * a.split_len;
+    if (lane == 0) {
+        mbar_init(&bar[warp], 1);
+        fence_mbar_init();
+        mbar_arrive_expect_tx(&bar[warp], static_cast<uint32_t>(len) * 16u);
+        bulk_g2s(sb, a.bodies + j0, static_cast<uint32_t>(len) * 16u, &bar[warp]);
+    }
+    __syncwarp();
+    mbar_wait(&bar[warp], 0);
+    const float eps2 = a.eps2;
+    for (int c0 = 0; c0 < len; c0 += kChunk) {
+        const int c1 = mn(len, c0 + kChunk);
+        it.chunk_begin();
+        if (c1 - c0 == kChunk) {
+#pragma unroll 4
+            for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
+        } else {
+            for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+        }
+        it.chunk_end();
+    }
+    part[warp * 32 + lane] = it.result(0);
+    __syncthreads();
+    if (warp == 0 && valid) {
+        float4 acc = part[lane];
+        for (int s = 1; s < a.splits; ++s) {
+            const float4 p = part[s * 32 + lane];
+            acc.x += p.x; acc.y += p.y; acc.z += p.z;
+        }
+        acc.w = 0.f;
+        a.accel[t] = acc;
+    }
+}
+
+static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
+    const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
+    static size_t attr = 0;
+    if (smem > attr) {
+        cudaError_t e = cudaFuncSetAttribute(force_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplits * 32 * 16));
+        if (e != cudaSuccess) return e;
+        attr = kSmallMaxSources * 16 + kMaxSplits * 32 * 16;
+    }
+    const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
+    force_small_kernel<<<static_cast<unsigned>(ctas), 32 * a.splits, smem, stream>>>(a);
+    return cudaGetLastError();
+}
+
 template <int BLOCK, int R>
 static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
@@ -290,6 +366,9 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
 
     const LaunchOverride& ov = launch_override();
+    // n_src <= kSmallMaxSources: in-CTA splits (same arithmetic and order, see force_small_kernel);
+    // a block_threads / per_thread override selects the general kernel (used by the bit-identity test).
+    if (n_src <= kSmallMaxSources && ov.block_threads == 0 && ov.per_thread == 0) return launch_small(a, stream);
     int block = ov.block_threads, R = ov.per_thread;
     if (block == 0 || R == 0) {
         // Automatic (tools/tune_nbody.py sweep on B200, profiles/tune_nbody_r01.jsonl): 256 threads x
