@@ -102,6 +102,15 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
  * Launch override: grid ignored; block_threads in {128, 256}; per_thread in {1, 2, 4, 8}.
  * =========================================================================== */
 size_t lime_map_nbody_workspace_bytes(int64_t n_src, int64_t tgt_count);
+/* Staging ablation (the paper's Fig. 8 memory-mapping variants, L391-398,
+ * and "any of the optimizations [can] be enabled and disabled", L212-216): selects, for the
+ * following lime_map_nbody calls on this thread, where the broadcast source array is read from:
+ * 0 = production kernels (TMA-staged shared memory), 1 = global scalar loads, 2 = global 128-bit
+ * loads, 3 = read-only (non-coherent) 128-bit loads, 4 = shared memory copied by threads, scalar
+ * reads, 5 = shared memory copied by threads, 128-bit reads, 6 = __constant__ memory (n_src <=
+ * 4096; includes a 64-KB device-to-device copy per call). Results are bit-identical for every
+ * variant. Returns LIME_ERR_INVALID_ARG for an unknown variant. */
+int lime_set_nbody_variant(int variant);
 int lime_nbody_splits(int64_t n_src);
 lime_status lime_map_nbody(const float *bodies, int64_t n_src, int64_t tgt_begin,
                            int64_t tgt_count, float eps2, float *accel,

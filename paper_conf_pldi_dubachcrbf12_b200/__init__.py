@@ -48,6 +48,7 @@ SIGNATURES = {
     "lime_num_sms": (_int, []),
     "lime_set_launch_override": (None, [_int, _int, _int]),
     "lime_map_nbody_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_set_nbody_variant": (_int, [_int]),
     "lime_nbody_splits": (_int, [_i64]),
     "lime_map_nbody": (_int, [_p, _i64, _i64, _i64, _f, _p, _p, _sz, _p]),
     "lime_map_nbody_integrate": (_int, [_p, _p, _p, _i64, _f, _p]),
@@ -126,6 +127,21 @@ def launch_override(grid_ctas: int = 0, block_threads: int = 0, per_thread: int 
         yield
     finally:
         L.lime_set_launch_override(0, 0, 0)
+
+
+NBODY_VARIANTS = {0: "tma_smem (production)", 1: "global_scalar", 2: "global_vec", 3: "readonly_vec",
+                  4: "local_scalar", 5: "local_vec", 6: "constant_vec"}
+
+
+@contextlib.contextmanager
+def nbody_variant(variant: int):
+    """Select the N-Body staging variant (F1 ablation, Fig. 8) on this thread."""
+    L = load()
+    _check(L.lime_set_nbody_variant(variant), "lime_set_nbody_variant")
+    try:
+        yield
+    finally:
+        L.lime_set_nbody_variant(0)
 
 
 def num_sms() -> int:

@@ -16,8 +16,10 @@ namespace lime {
 
 static thread_local char g_last_error[512] = "";
 static thread_local LaunchOverride g_override;
+static thread_local int g_nbody_variant = 0;
 
 const LaunchOverride& launch_override() { return g_override; }
+int nbody_variant() { return g_nbody_variant; }
 
 int device_num_sms() {
     static int cached[64] = {0};
@@ -122,6 +124,12 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread) 
     g_override.grid_ctas = grid_ctas > 0 ? grid_ctas : 0;
     g_override.block_threads = block_threads > 0 ? block_threads : 0;
     g_override.per_thread = per_thread > 0 ? per_thread : 0;
+}
+
+int lime_set_nbody_variant(int variant) {
+    if (variant < 0 || variant > 6) return LIME_ERR_INVALID_ARG;
+    g_nbody_variant = variant;
+    return LIME_OK;
 }
 
 // ============================================================================== N-Body

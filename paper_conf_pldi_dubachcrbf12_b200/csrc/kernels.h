@@ -13,6 +13,7 @@ struct LaunchOverride {
     int per_thread = 0;
 };
 const LaunchOverride& launch_override();
+int nbody_variant();   // staging ablation selector (0 = production kernels), see lime_set_nbody_variant
 int device_num_sms();
 
 // ------------------------------------------------------------------ N-Body

@@ -163,6 +163,49 @@ struct Interact<R, true> {
     }
 };
 
+// Output (A7: float4 stores) and split combine (A8), shared by every force-kernel variant: with
+// S > 1, each CTA writes its split partials, and the last CTA of a target tile (atomic ticket)
+// adds the S partials in split order and resets the ticket.
+template <int BLOCK, int R, class IT>
+__device__ __forceinline__ void finish_targets(const ForceArgs& a, const IT& it, const bool (&valid)[R], int tile,
+                                               int split, int64_t tbase, int* s_last) {
+    if (a.splits == 1) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+            if (valid[r]) a.accel[t] = it.result(r);
+        }
+        return;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        if (valid[r]) __stcg(a.partial + static_cast<int64_t>(split) * a.tgt_count + t, it.result(r));
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned prev = atomicAdd(a.counters + tile, 1u);
+        *s_last = (prev == static_cast<unsigned>(a.splits - 1));
+    }
+    __syncthreads();
+    if (!*s_last) return;
+    __threadfence();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        if (!valid[r]) continue;
+        float4 acc = __ldcg(a.partial + t);
+        for (int s = 1; s < a.splits; ++s) {
+            const float4 p = __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
+            acc.x += p.x; acc.y += p.y; acc.z += p.z;
+        }
+        acc.w = 0.f;
+        a.accel[t] = acc;
+    }
+    if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
+}
+
 template <int BLOCK, int R, bool kPacked>
 __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ ForceArgs a) {
     __shared__ __align__(128) float4 sbuf[2][kTileJ];
@@ -227,42 +270,7 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
         if (threadIdx.x == 0 && t + 2 < ntiles) issue(t + 2);
     }
 
-    // ---- output (A7: float4 stores) / split combine (A8)
-    if (a.splits == 1) {
-#pragma unroll
-        for (int r = 0; r < R; ++r) {
-            const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
-            if (valid[r]) a.accel[t] = it.result(r);
-        }
-        return;
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
-        if (valid[r]) __stcg(a.partial + static_cast<int64_t>(split) * a.tgt_count + t, it.result(r));
-    }
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        const unsigned prev = atomicAdd(a.counters + tile, 1u);
-        s_last = (prev == static_cast<unsigned>(a.splits - 1));
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
-        if (!valid[r]) continue;
-        float4 acc = __ldcg(a.partial + t);
-        for (int s = 1; s < a.splits; ++s) {
-            const float4 p = __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
-            acc.x += p.x; acc.y += p.y; acc.z += p.z;
-        }
-        acc.w = 0.f;
-        a.accel[t] = acc;
-    }
-    if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
+    finish_targets<BLOCK, R>(a, it, valid, tile, split, tbase, &s_last);
 }
 
 // =====================================================================================
@@ -341,6 +349,109 @@ static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
     return cudaGetLastError();
 }
 
+// =====================================================================================
+// Staging ablation (the paper's Fig. 8: the same kernel with the
+// broadcast array mapped to global, local, texture or constant memory, with or without
+// vectorisation; L212-216: every optimisation can be switched off for automated exploration).
+// Same arithmetic and summation order as force_kernel, so every variant is bit-identical; only
+// where the source bodies come from changes:
+//   1 global, scalar     4 x ld.global.f32 per body (L1-cached)
+//   2 global, vector     ld.global.v4.f32 per body
+//   3 read-only, vector  ld.global.nc.v4.f32 (the image/texture path's B200 equivalent)
+//   4 local, scalar      threads copy a 1024-body tile into SoA shared arrays; 4 x LDS.32 per body
+//   5 local, vector      threads copy the tile with LDG.128/STS.128; LDS.128 per body
+//   6 constant, vector   bodies in __constant__ memory (n_src <= 4096 = 64 KB, Table 2's size)
+// (variant 0 = force_kernel: 1-D TMA bulk copies into a double-buffered smem ring). Broadcast
+// reads make every smem variant bank-conflict free, so the paper's padding variant has no B200
+// counterpart here.
+// =====================================================================================
+constexpr int kConstBodies = 4096;
+__constant__ float4 c_bodies[kConstBodies];
+
+template <int BLOCK, int R, int V>
+__global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_constant__ ForceArgs a) {
+    constexpr bool kPacked = (R % 2 == 0);
+    __shared__ __align__(128) float4 tile4[(V == 5) ? kTileJ : 1];
+    __shared__ float tx[(V == 4) ? kTileJ : 1], ty[(V == 4) ? kTileJ : 1], tz[(V == 4) ? kTileJ : 1],
+        tm[(V == 4) ? kTileJ : 1];
+    __shared__ int s_last;
+    const int tile = blockIdx.x;
+    const int split = blockIdx.y;
+    const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * R);
+    Interact<R, kPacked> it;
+    bool valid[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
+        valid[r] = t < a.tgt_count;
+        it.set(r, __ldg(a.bodies + a.tgt_begin + (valid[r] ? t : a.tgt_count - 1)));
+    }
+    it.zero_all();
+    const int64_t j0 = static_cast<int64_t>(split) * a.split_len;
+    const int64_t j1 = mn<int64_t>(a.n_src, j0 + a.split_len);
+    const float eps2 = a.eps2;
+    const float* bf = reinterpret_cast<const float*>(a.bodies);
+    for (int64_t tb = j0; tb < j1; tb += kTileJ) {
+        const int len = static_cast<int>(mn<int64_t>(kTileJ, j1 - tb));
+        if (V == 4 || V == 5) {
+            __syncthreads();
+            for (int k = threadIdx.x; k < len; k += BLOCK) {
+                const float4 b = a.bodies[tb + k];
+                if (V == 5) tile4[k] = b;
+                else { tx[k] = b.x; ty[k] = b.y; tz[k] = b.z; tm[k] = b.w; }
+            }
+            __syncthreads();
+        }
+        auto src = [&](int j) -> float4 {
+            const int64_t g = tb + j;
+            if constexpr (V == 1) return make_float4(bf[4 * g], bf[4 * g + 1], bf[4 * g + 2], bf[4 * g + 3]);
+            else if constexpr (V == 2) {
+                float4 v;
+                asm volatile("ld.global.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(a.bodies + g));
+                return v;
+            } else if constexpr (V == 3) return __ldg(a.bodies + g);
+            else if constexpr (V == 4) return make_float4(tx[j], ty[j], tz[j], tm[j]);
+            else if constexpr (V == 5) return tile4[j];
+            else return c_bodies[g];
+        };
+        for (int c0 = 0; c0 < len; c0 += kChunk) {
+            const int c1 = mn(len, c0 + kChunk);
+            it.chunk_begin();
+            if (c1 - c0 == kChunk) {
+#pragma unroll 4
+                for (int j = c0; j < c0 + kChunk; ++j) it.body(src(j), eps2);
+            } else {
+                for (int j = c0; j < c1; ++j) it.body(src(j), eps2);
+            }
+            it.chunk_end();
+        }
+    }
+    finish_targets<BLOCK, R>(a, it, valid, tile, split, tbase, &s_last);
+}
+
+template <int BLOCK, int R>
+static cudaError_t launch_ablate(const ForceArgs& a, int v, cudaStream_t stream) {
+    const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
+    dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
+    switch (v) {
+        case 1: force_ablate_kernel<BLOCK, R, 1><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 2: force_ablate_kernel<BLOCK, R, 2><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 3: force_ablate_kernel<BLOCK, R, 3><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 4: force_ablate_kernel<BLOCK, R, 4><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 5: force_ablate_kernel<BLOCK, R, 5><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 6: {
+            if (a.n_src > kConstBodies) return cudaErrorInvalidValue;
+            cudaError_t e = cudaMemcpyToSymbolAsync(c_bodies, a.bodies, static_cast<size_t>(a.n_src) * 16, 0,
+                                                    cudaMemcpyDeviceToDevice, stream);
+            if (e != cudaSuccess) return e;
+            force_ablate_kernel<BLOCK, R, 6><<<grid, BLOCK, 0, stream>>>(a);
+            break;
+        }
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
 template <int BLOCK, int R>
 static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
@@ -366,6 +477,12 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
 
     const LaunchOverride& ov = launch_override();
+    if (nbody_variant() != 0) {                       // F1 staging ablation (general mapping only)
+        const int v = nbody_variant();
+        if (ov.block_threads == 128 && ov.per_thread == 1) return launch_ablate<128, 1>(a, v, stream);
+        if (ov.block_threads == 128) return launch_ablate<128, 2>(a, v, stream);
+        return launch_ablate<256, 2>(a, v, stream);
+    }
     // n_src <= kSmallMaxSources: in-CTA splits (same arithmetic and order, see force_small_kernel);
     // a block_threads / per_thread override selects the general kernel (used by the bit-identity test).
     if (n_src <= kSmallMaxSources && ov.block_threads == 0 && ov.per_thread == 0) return launch_small(a, stream);

@@ -121,3 +121,16 @@ def test_errors_surface_as_exceptions(lime):
         lime.map_nbody(b, 0.0)
     with pytest.raises(lime.LimeError, match="INVALID_ARG"):
         lime.map_nbody(b, 1e-4, 10, 7)
+
+
+@pytest.mark.parametrize("n,count", [(4096, 4096), (3000, 1000), (1 << 17, 1 << 12)])
+def test_staging_ablation_variants_bit_identical(lime, n, count):
+    # F1 (Fig. 8): every memory-mapping variant computes the same sums in the same order
+    b = _dev(inputs.nbody_bodies(n, seed=21))
+    ref = lime.map_nbody(b, float(EPS2), 0, count).cpu()
+    for v in range(1, 7):
+        if v == 6 and n > 4096:
+            continue
+        with lime.nbody_variant(v):
+            got = lime.map_nbody(b, float(EPS2), 0, count).cpu()
+        assert torch.equal(got, ref), v
