@@ -65,6 +65,8 @@ def _declare(L):
         "oracle_mandelbrot": (None, [_i32, _i32, _i32, _i32, _i32, _f, _f, _f, _f, _i32, _p]),
         "oracle_matmul_bf16": (None, [_p, _p, _i64, _i64, _i64, _p]),
         "oracle_matmul_bf16_entries": (None, [_p, _p, _i64, _p, _p, _i64, _p, _p]),
+        "oracle_coulomb_potential": (None, [_p, _i64, _i32, _i32, _i32, _f, _f, _p, _p]),
+        "oracle_mriq": (None, [_p, _i64, _p, _i64, _p, _p]),
         "oracle_reduce_sum_f32": (_d, [_p, _i64]),
         "oracle_reduce_sum_f64": (_d, [_p, _i64]),
         "oracle_reduce_sum_i32": (_i32, [_p, _i64]),
@@ -216,6 +218,41 @@ def matmul_bf16_entries(A_bits, Bt_bits, rows, cols, threads: int = 1):
 
     _parallel(work, n, threads, chunked=True)
     return Cv, Av
+
+
+# ------------------------------------------------------------ Parboil CP / MRI-Q
+def coulomb_potential(atoms, nx: int, ny: int, z: float, h: float, iy0: int = 0, threads: int = 1):
+    """oracle_coulomb_potential: V double [ny][nx] for lattice rows iy0..iy0+ny-1, and
+    sum_j |q_j| / r_j; `threads` splits the rows (each part is the single-threaded C loop)."""
+    a = _c(atoms, np.float32).reshape(-1, 4)
+    V = np.zeros((ny, nx), dtype=np.float64)
+    M = np.zeros((ny, nx), dtype=np.float64)
+    L = lib()
+
+    def work(lo, hi):
+        if hi > lo:
+            L.oracle_coulomb_potential(a.ctypes.data, a.shape[0], nx, iy0 + lo, hi - lo, float(z), float(h),
+                                       V[lo:hi].ctypes.data, M[lo:hi].ctypes.data)
+
+    _parallel(work, ny, threads)
+    return V, M
+
+
+def mriq(kspace, voxels, threads: int = 1):
+    """oracle_mriq: (Qr, Qi) double [X][2] and sum_k phiMag_k [X]."""
+    ks = _c(kspace, np.float32).reshape(-1, 5)
+    vx = _c(voxels, np.float32).reshape(-1, 3)
+    out = np.zeros((vx.shape[0], 2), dtype=np.float64)
+    mag = np.zeros(vx.shape[0], dtype=np.float64)
+    L = lib()
+
+    def work(lo, hi):
+        if hi > lo:
+            L.oracle_mriq(ks.ctypes.data, ks.shape[0], vx[lo:hi].ctypes.data, hi - lo,
+                          out[lo:hi].ctypes.data, mag[lo:hi].ctypes.data)
+
+    _parallel(work, vx.shape[0], threads)
+    return out, mag
 
 
 # ------------------------------------------------------------- Reductions

@@ -388,3 +388,70 @@ int64_t oracle_reduce_max_i64(const int64_t *x, int64_t n)
     for (int64_t i = 0; i < n; ++i) if (x[i] > m) m = x[i];
     return m;
 }
+
+/* ------------------------------------------------------------------------
+ * Parboil-CP: Coulombic potential on one lattice slice (Table 3,
+ * "Parboil-CP Coulombic Potential 62KB -> 1MB Float"). The
+ * paper describes only the benchmark name and sizes; reading DESIGN.md R12:
+ * direct Coulomb summation
+ *   V[iy][ix] = sum_j q_j / sqrt((x - x_j)^2 + (y - y_j)^2 + (z - z_j)^2),
+ *   x = fl32(ix * h), y = fl32(iy * h)  (grid coordinates are the fp32 products),
+ * evaluated in double from the fp32 inputs, sequential j, for lattice rows
+ * iy0 .. iy0+ny-1 (out/mag are [ny][nx]). atoms is [n][4] (x, y, z, q). If
+ * mag != NULL it receives sum_j |q_j| / r_j. */
+void oracle_coulomb_potential(const float *atoms, int64_t n_atoms, int32_t nx, int32_t iy0, int32_t ny,
+                              float z, float h, double *out, double *mag)
+{
+    oracle_fp_env();
+    for (int32_t r = 0; r < ny; ++r) {
+        const int32_t iy = iy0 + r;
+        const float yf = (float)iy * h;
+        for (int32_t ix = 0; ix < nx; ++ix) {
+            const float xf = (float)ix * h;
+            double v = 0.0, m = 0.0;
+            for (int64_t j = 0; j < n_atoms; ++j) {
+                const double dx = (double)xf - (double)atoms[4 * j + 0];
+                const double dy = (double)yf - (double)atoms[4 * j + 1];
+                const double dz = (double)z - (double)atoms[4 * j + 2];
+                const double r = sqrt(dx * dx + dy * dy + dz * dz);
+                v += (double)atoms[4 * j + 3] / r;
+                m += fabs((double)atoms[4 * j + 3]) / r;
+            }
+            out[(int64_t)r * nx + ix] = v;
+            if (mag) mag[(int64_t)r * nx + ix] = m;
+        }
+    }
+}
+
+/* ------------------------------------------------------------------------
+ * Parboil-MRI-Q: the Q matrix of non-Cartesian MRI reconstruction (PAPER.md
+ * Table 3, "Parboil-MRIQ Magnetic Resonance Imaging 432KB -> 256KB
+ * Float"). Reading DESIGN.md R13 (Parboil's definition):
+ *   phiMag_k = phiR_k^2 + phiI_k^2
+ *   Qr(x) = sum_k phiMag_k cos(2 pi (kx_k x + ky_k y + kz_k z))
+ *   Qi(x) = sum_k phiMag_k sin(2 pi (kx_k x + ky_k y + kz_k z))
+ * in double from the fp32 inputs, sequential k. kspace is [K][5] floats
+ * (kx, ky, kz, phiR, phiI); voxels is [X][3] (x, y, z); out is [X][2]
+ * (Qr, Qi). If mag != NULL it receives sum_k phiMag_k. */
+void oracle_mriq(const float *kspace, int64_t n_k, const float *voxels, int64_t n_x, double *out,
+                 double *mag)
+{
+    oracle_fp_env();
+    const double two_pi = 6.283185307179586476925286766559;
+    for (int64_t i = 0; i < n_x; ++i) {
+        const double x = voxels[3 * i + 0], y = voxels[3 * i + 1], zz = voxels[3 * i + 2];
+        double qr = 0.0, qi = 0.0, m = 0.0;
+        for (int64_t k = 0; k < n_k; ++k) {
+            const double pr = kspace[5 * k + 3], pi = kspace[5 * k + 4];
+            const double phimag = pr * pr + pi * pi;
+            const double arg = two_pi * ((double)kspace[5 * k + 0] * x + (double)kspace[5 * k + 1] * y +
+                                         (double)kspace[5 * k + 2] * zz);
+            qr += phimag * cos(arg);
+            qi += phimag * sin(arg);
+            m += phimag;
+        }
+        out[2 * i + 0] = qr;
+        out[2 * i + 1] = qi;
+        if (mag) mag[i] = m;
+    }
+}

@@ -132,3 +132,41 @@ def reduce_array(n: int, dtype: str, seed: int = 6) -> np.ndarray:
     if dtype == "i64":
         return (raw >> np.uint64(23)).astype(np.int64) - (1 << 40)
     raise ValueError(dtype)
+
+
+# ------------------------------------------------- Parboil CP / MRI-Q (SURVEY.md §8(f) F2)
+CP_NX = CP_NY = 512        # Table 3: 1 MB float output = 512 x 512 (L353)
+CP_ATOMS = 3968            # Table 3: 62 KB float4 input ~ 3968 atoms (L353)
+CP_H = 0.1                 # lattice spacing (Parboil CP's default grid spacing)
+CP_Z = 25.6                # slice through the middle of the 51.2-wide box
+
+
+def cp_atoms(n: int = CP_ATOMS, seed: int = 7, box: float = CP_NX * CP_H) -> np.ndarray:
+    """[n][4] float32 (x, y, z, q): positions U[0, box)^3, charges U[-1, 1)."""
+    out = np.empty((n, 4), dtype=np.float32)
+    for c in range(3):
+        out[:, c] = (box * uniform24(seed, c, n).astype(np.float64)).astype(np.float32)
+    out[:, 3] = (2.0 * uniform24(seed, 3, n).astype(np.float64) - 1.0).astype(np.float32)
+    return out
+
+
+MRIQ_VOXELS = 32768        # Table 3: 256 KB float output = 32768 x (Qr, Qi) (L353-354)
+MRIQ_K = 3072              # Table 3: 432 KB input = 32768 x 3 floats + 3072 x (kx, ky, kz, phiR) ...
+
+
+def mriq_kspace(n: int = MRIQ_K, seed: int = 8) -> np.ndarray:
+    """[n][5] float32 (kx, ky, kz, phiR, phiI): k U[-32, 32)^3, phi U[-1, 1)^2."""
+    out = np.empty((n, 5), dtype=np.float32)
+    for c in range(3):
+        out[:, c] = (64.0 * uniform24(seed, c, n).astype(np.float64) - 32.0).astype(np.float32)
+    for c in (3, 4):
+        out[:, c] = (2.0 * uniform24(seed, c, n).astype(np.float64) - 1.0).astype(np.float32)
+    return out
+
+
+def mriq_voxels(n: int = MRIQ_VOXELS, seed: int = 9) -> np.ndarray:
+    """[n][3] float32 (x, y, z): U[-0.5, 0.5)^3."""
+    out = np.empty((n, 3), dtype=np.float32)
+    for c in range(3):
+        out[:, c] = (uniform24(seed, c, n).astype(np.float64) - 0.5).astype(np.float32)
+    return out

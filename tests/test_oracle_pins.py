@@ -347,3 +347,107 @@ def test_reduce_empty_identity():
     assert oracle.reduce("max", e["f64"], "f64") == -math.inf
     assert oracle.reduce("min", e["i32"], "i32") == 2**31 - 1
     assert oracle.reduce("max", e["i64"], "i64") == -(2**63)
+
+
+# =============================================== Parboil CP (F2, Table 3)
+# oracle_coulomb_potential: direct Coulomb summation on a lattice slice; reading R12
+
+def test_cp_point_charge_values():
+    # q = 2 at (3, 4, 0) seen from the lattice origin (z = 0): V = 2 / 5; at (ix=1): d = sqrt(4+16)
+    atoms = np.array([[3.0, 4.0, 0.0, 2.0]], dtype=np.float32)
+    V, M = oracle.coulomb_potential(atoms, 2, 1, 0.0, 1.0)
+    assert V[0, 0] == 0.4 and V[0, 1] == 2.0 / math.sqrt(20.0)
+    assert np.array_equal(M, np.abs(V))
+
+
+def test_cp_superposition_and_sign():
+    a = inputs.cp_atoms(40, seed=3, box=5.0)
+    b = inputs.cp_atoms(25, seed=4, box=5.0)
+    Va, _ = oracle.coulomb_potential(a, 9, 7, 2.05, 0.5)
+    Vb, _ = oracle.coulomb_potential(b, 9, 7, 2.05, 0.5)
+    Vab, _ = oracle.coulomb_potential(np.concatenate([a, b]), 9, 7, 2.05, 0.5)
+    np.testing.assert_allclose(Vab, Va + Vb, rtol=1e-13, atol=1e-13)
+    pos = a.copy(); pos[:, 3] = np.abs(pos[:, 3])
+    assert np.all(oracle.coulomb_potential(pos, 9, 7, 2.05, 0.5)[0] > 0)    # positive charges
+
+
+def test_cp_mean_value_property():
+    # harmonic away from charges (Laplace's equation): the 6-point stencil mean minus the centre
+    # value vanishes like h^4 (the h^2 term is the Laplacian, which is 0); a wrong power of r
+    # (e.g. 1/r^2) leaves a nonzero Laplacian and an h^2 decay.
+    atoms = np.array([[0.3, -0.2, 0.1, 1.0], [-0.4, 0.5, -0.3, -0.7]], dtype=np.float32)
+    def lap(h):
+        pts = np.array([[3, 3, 3], [3 + h, 3, 3], [3 - h, 3, 3], [3, 3 + h, 3], [3, 3 - h, 3], [3, 3, 3 + h], [3, 3, 3 - h]])
+        v = []
+        for p in pts:   # lattice origin at the point: shift atoms by -p (exact in double for these values)
+            sh = atoms.copy().astype(np.float64); sh[:, :3] -= p
+            v.append(oracle.coulomb_potential(sh.astype(np.float32), 1, 1, 0.0, 1.0)[0][0, 0])
+        v = np.array(v)
+        return abs(v[1:].mean() - v[0]) / abs(v[0])
+    l4, l2, l1 = lap(0.4), lap(0.2), lap(0.1)
+    assert l4 < 1e-4 and l2 < l4 / 10 and l1 < l2 / 10
+
+
+def test_cp_dipole_far_field():
+    # charges +q, -q at +-s/2 on z: far along z at distance r, V ~ q s / r^2 (textbook multipole)
+    q, s, r = 1.0, 0.01, 10.0
+    atoms = np.array([[0, 0, s / 2, q], [0, 0, -s / 2, -q]], dtype=np.float32)
+    V, _ = oracle.coulomb_potential(atoms, 1, 1, r, 1.0)
+    assert abs(V[0, 0] - q * s / r**2) <= 1e-3 * q * s / r**2
+
+
+def test_cp_numpy_brute_force():
+    atoms = inputs.cp_atoms(50, seed=5, box=3.2)
+    V, M = oracle.coulomb_potential(atoms, 32, 8, 1.55, 0.1, iy0=5)
+    xs = (np.arange(32, dtype=np.float32) * np.float32(0.1)).astype(np.float64)
+    ys = (np.arange(5, 13, dtype=np.float32) * np.float32(0.1)).astype(np.float64)
+    a = atoms.astype(np.float64)
+    d = np.sqrt((xs[None, :, None] - a[None, None, :, 0]) ** 2 + (ys[:, None, None] - a[None, None, :, 1]) ** 2
+                + (float(np.float32(1.55)) - a[None, None, :, 2]) ** 2)
+    np.testing.assert_allclose(V, (a[:, 3] / d).sum(-1), rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(M, (np.abs(a[:, 3]) / d).sum(-1), rtol=1e-12)
+
+
+# ============================================ Parboil MRI-Q (F2, Table 3)
+# oracle_mriq: Qr/Qi = sum_k |phi_k|^2 (cos, sin)(2 pi k.x); reading R13
+
+def test_mriq_dc_sample_and_odd_symmetry():
+    ks = np.array([[0, 0, 0, 0.6, 0.8]], dtype=np.float32)          # k = 0, |phi|^2 = 1
+    vx = inputs.mriq_voxels(10, seed=1)
+    Q, M = oracle.mriq(ks, vx)
+    assert np.allclose(Q[:, 0], 1.0, atol=1e-15) and np.all(Q[:, 1] == 0.0) and np.allclose(M, 1.0)
+    k = inputs.mriq_kspace(20, seed=2)
+    kk = np.concatenate([k, k * np.array([-1, -1, -1, 1, 1], dtype=np.float32)])   # +-k, same phi
+    Q2, _ = oracle.mriq(kk, vx)
+    assert np.abs(Q2[:, 1]).max() <= 1e-12                               # sin is odd
+    Q1, _ = oracle.mriq(k, vx)
+    np.testing.assert_allclose(Q2[:, 0], 2 * Q1[:, 0], rtol=1e-12, atol=1e-12)   # cos is even
+
+
+def test_mriq_integer_phase_and_bound():
+    ks = np.array([[1, 2, 3, 1.0, 0.0], [-2, 1, 0, 0.5, 0.5]], dtype=np.float32)
+    vx = np.array([[1, 0, 0], [0, 1, 0], [1, 1, 1], [-2, 3, 1]], dtype=np.float32)    # k.x integers
+    Q, M = oracle.mriq(ks, vx)
+    np.testing.assert_allclose(Q[:, 0], M, rtol=0, atol=1e-12)
+    np.testing.assert_allclose(Q[:, 1], 0.0, atol=1e-12)
+    k = inputs.mriq_kspace(64, seed=3)
+    Qr, Mr = oracle.mriq(k, inputs.mriq_voxels(50, seed=4))
+    assert np.all(np.hypot(Qr[:, 0], Qr[:, 1]) <= Mr * (1 + 1e-12))
+
+
+def test_mriq_shift_theorem_and_brute_force():
+    k = inputs.mriq_kspace(1, seed=5)
+    vx = inputs.mriq_voxels(16, seed=6)
+    Q, _ = oracle.mriq(k, vx)
+    z = Q[:, 0] + 1j * Q[:, 1]
+    kv = k[0, :3].astype(np.float64)
+    phase = np.exp(2j * np.pi * (vx.astype(np.float64) @ kv))
+    np.testing.assert_allclose(z, (k[0, 3].astype(np.float64) ** 2 + k[0, 4].astype(np.float64) ** 2) * phase, rtol=1e-12)
+    kk = inputs.mriq_kspace(37, seed=7)
+    vv = inputs.mriq_voxels(23, seed=8)
+    Q, M = oracle.mriq(kk, vv)
+    a = kk.astype(np.float64)
+    arg = 2 * np.pi * (vv.astype(np.float64) @ a[:, :3].T)
+    pm = a[:, 3] ** 2 + a[:, 4] ** 2
+    np.testing.assert_allclose(Q[:, 0], (pm * np.cos(arg)).sum(1), rtol=1e-11, atol=1e-11)
+    np.testing.assert_allclose(Q[:, 1], (pm * np.sin(arg)).sum(1), rtol=1e-11, atol=1e-11)
