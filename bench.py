@@ -348,6 +348,32 @@ def run_extras(peaks, flush):
     except lime.LimeError as e:
         out["matmul"] = {"workload": "configs[3]", "unavailable": str(e)}
 
+    # F2: Parboil-CP and MRI-Q at the paper's Table 3 sizes (L353-354); both are
+    # bound by the MUFU (XU) pipe: 1 rsqrt (CP) / 1 sin + 1 cos (MRI-Q) per interaction.
+    mufu_peak = 16.0 * SMS_B200 * SM_MAX_MHZ_NOMINAL * 1e6      # 16 lanes/clk/SM (microbench: 16.00)
+    atoms = torch.from_numpy(inputs.cp_atoms()).cuda()
+    npts = inputs.CP_NX * inputs.CP_NY
+    V = torch.empty(npts, device="cuda")
+    med, _ = time_launches(lambda: lime.map_coulomb(atoms, inputs.CP_NX, inputs.CP_NY, inputs.CP_Z, inputs.CP_H, out=V),
+                           30, 3, flush)
+    inter = float(npts) * atoms.shape[0]
+    out["parboil_cp"] = {"workload": "F2: Parboil-CP Coulombic potential, 3968 atoms x 512^2 lattice (Table 3)",
+                         "value": inter / (med * 1e-3), "unit": "interactions/s", "ms_per_launch": med,
+                         "roofline": {"bound": "alu", "achieved": inter / (med * 1e-3) / 1e12, "peak": mufu_peak / 1e12,
+                                      "unit": "T MUFU ops/s", "frac": inter / (med * 1e-3) / mufu_peak,
+                                      "traffic": ncu_traffic("parboil_cp")}}
+    k = torch.from_numpy(inputs.mriq_kspace()).cuda()
+    vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
+    Q = torch.empty((vx.shape[0], 2), device="cuda")
+    med, _ = time_launches(lambda: lime.map_mriq(k, vx, out=Q), 30, 3, flush)
+    inter = float(vx.shape[0]) * k.shape[0]
+    out["parboil_mriq"] = {"workload": "F2: Parboil-MRI-Q, 3072 k-samples x 32768 voxels (Table 3)",
+                           "value": inter / (med * 1e-3), "unit": "interactions/s", "ms_per_launch": med,
+                           "roofline": {"bound": "alu", "achieved": 2 * inter / (med * 1e-3) / 1e12,
+                                        "peak": mufu_peak / 1e12, "unit": "T MUFU ops/s",
+                                        "frac": 2 * inter / (med * 1e-3) / mufu_peak, "traffic": ncu_traffic("parboil_mriq")}}
+    del atoms, V, k, vx, Q
+
     # reduction `!`: sum over 2^28 fp32 (1 GiB)
     x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
     r = torch.empty((), dtype=torch.float32, device="cuda")

@@ -191,6 +191,39 @@ lime_status lime_map_matmul_bf16(const uint16_t *A, const uint16_t *Bt, float *C
                                  int64_t N, int64_t K, void *stream);
 
 /* ===========================================================================
+ * Parboil-CP: Coulombic potential on one lattice slice (Table 3;
+ * SURVEY.md §8(f) F2; definition DESIGN.md R12): a map over lattice points with
+ * the atom array as broadcast operand,
+ *   V[t] = sum_j q_j / |p_t - r_j|,  t = p_begin + k (k in [0, p_count)),
+ *   p_t = (fl32(ix h), fl32(iy h), z), ix = t % nx, iy = t / nx.
+ * atoms [n_atoms][4] float (x, y, z, q), 16-B aligned; V [p_count] float, must
+ * not overlap atoms. nx, ny >= 1; 0 <= p_begin <= p_begin + p_count <= nx*ny;
+ * h > 0 and z finite. A lattice point exactly on an atom gives inf (no
+ * softening, as in Parboil). Sum order: 256-atom chunks, split partials,
+ * split order (deterministic, launch- and shard-independent).
+ * ws: lime_map_coulomb_workspace_bytes(n_atoms, p_count) bytes, zeroed once.
+ * =========================================================================== */
+size_t lime_map_coulomb_workspace_bytes(int64_t n_atoms, int64_t p_count);
+lime_status lime_map_coulomb(const float *atoms, int64_t n_atoms, int32_t nx, int32_t ny, int64_t p_begin,
+                             int64_t p_count, float z, float h, float *V, void *ws, size_t ws_bytes,
+                             void *stream);
+
+/* ===========================================================================
+ * Parboil-MRI-Q (Table 3; definition
+ * DESIGN.md R13): a map over voxels with the k-space samples as broadcast
+ * operand, Q[i] = (Qr, Qi) = sum_k |phi_k|^2 (cos, sin)(2 pi k.x_i),
+ * i = x_begin + m (m in [0, x_count)).
+ * kspace [n_k][5] float (kx, ky, kz, phiR, phiI); voxels [n_x][3] float; Q
+ * [x_count][2] float, 8-B aligned, must not overlap the inputs. The phase is
+ * reduced to [-1/2, 1/2] turn before the (MUFU) sine/cosine, so |k.x| must
+ * stay below 2^22 turns. ws: lime_map_mriq_workspace_bytes(n_k, x_count) bytes
+ * (holds the (kx, ky, kz, |phi|^2) table and the split partials), zeroed once.
+ * =========================================================================== */
+size_t lime_map_mriq_workspace_bytes(int64_t n_k, int64_t x_count);
+lime_status lime_map_mriq(const float *kspace, int64_t n_k, const float *voxels, int64_t n_x, int64_t x_begin,
+                          int64_t x_count, float *Q, void *ws, size_t ws_bytes, void *stream);
+
+/* ===========================================================================
  * Reductions `!` over an array x[n] (L160-163; L188-189 "the compiler may
  * infer a parallel reduction"; R9). Tree: per-thread fold ->
  * warp shuffle -> CTA -> last CTA combines the CTA partials in index order.

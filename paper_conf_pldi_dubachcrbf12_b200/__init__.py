@@ -60,6 +60,10 @@ SIGNATURES = {
     "lime_map_mandelbrot": (_int, [_i32, _i32, _i32, _i32, _i32, _f, _f, _f, _f, _i32, _p, _p, _sz, _p]),
     "lime_map_matmul_bf16": (_int, [_p, _p, _p, _i64, _i64, _i64, _p]),
     "lime_reduce_workspace_bytes": (_sz, []),
+    "lime_map_coulomb_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_map_coulomb": (_int, [_p, _i64, _i32, _i32, _i64, _i64, _f, _f, _p, _p, _sz, _p]),
+    "lime_map_mriq_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_map_mriq": (_int, [_p, _i64, _p, _i64, _i64, _i64, _p, _p, _sz, _p]),
 }
 for _op in ("sum", "min", "max"):
     for _dt in ("f32", "f64", "i32", "i64"):
@@ -248,6 +252,37 @@ def map_matmul_bf16(A: torch.Tensor, Bt: torch.Tensor, out=None) -> torch.Tensor
     out = torch.empty((M, N), dtype=torch.float32, device=A.device) if out is None else out
     _check(L.lime_map_matmul_bf16(A.data_ptr(), Bt.data_ptr(), out.data_ptr(), M, N, K, _stream(A.device)),
            "lime_map_matmul_bf16")
+    return out
+
+
+# --------------------------------------------------------- Parboil CP / MRI-Q (F2)
+def map_coulomb(atoms: torch.Tensor, nx: int, ny: int, z: float, h: float, p_begin: int = 0,
+                p_count: int | None = None, out=None) -> torch.Tensor:
+    """Coulombic potential V[p] over lattice points [p_begin, p_begin+p_count) of an nx x ny slice."""
+    L = load()
+    _dev_tensor(atoms, torch.float32, "atoms", 4)
+    if p_count is None:
+        p_count = nx * ny - p_begin
+    out = torch.empty(max(p_count, 0), dtype=torch.float32, device=atoms.device) if out is None else out
+    ws = workspace(atoms.device, "coulomb", L.lime_map_coulomb_workspace_bytes(atoms.shape[0], max(p_count, 0)))
+    _check(L.lime_map_coulomb(atoms.data_ptr(), atoms.shape[0], nx, ny, p_begin, p_count, z, h, out.data_ptr(),
+                              ws.data_ptr(), ws.numel(), _stream(atoms.device)), "lime_map_coulomb")
+    return out
+
+
+def map_mriq(kspace: torch.Tensor, voxels: torch.Tensor, x_begin: int = 0, x_count: int | None = None,
+             out=None) -> torch.Tensor:
+    """MRI-Q: (Qr, Qi) [x_count][2] for voxels [x_begin, x_begin+x_count)."""
+    L = load()
+    _dev_tensor(kspace, torch.float32, "kspace", 5)
+    _dev_tensor(voxels, torch.float32, "voxels", 3)
+    n_x = voxels.shape[0]
+    if x_count is None:
+        x_count = n_x - x_begin
+    out = torch.empty((max(x_count, 0), 2), dtype=torch.float32, device=voxels.device) if out is None else out
+    ws = workspace(voxels.device, "mriq", L.lime_map_mriq_workspace_bytes(kspace.shape[0], max(x_count, 0)))
+    _check(L.lime_map_mriq(kspace.data_ptr(), kspace.shape[0], voxels.data_ptr(), n_x, x_begin, x_count,
+                           out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(voxels.device)), "lime_map_mriq")
     return out
 
 

@@ -291,6 +291,59 @@ lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first
                     "lime_map_mandelbrot");
 }
 
+// ======================================================================= Parboil CP / MRI-Q
+size_t lime_map_coulomb_workspace_bytes(int64_t n_atoms, int64_t p_count) {
+    if (n_atoms < 0 || p_count < 0) return 0;
+    return parboil::cp_workspace_bytes(n_atoms, p_count);
+}
+
+lime_status lime_map_coulomb(const float* atoms, int64_t n_atoms, int32_t nx, int32_t ny, int64_t p_begin,
+                             int64_t p_count, float z, float h, float* V, void* ws, size_t ws_bytes, void* stream) {
+    const int64_t np = static_cast<int64_t>(nx) * ny;
+    if (n_atoms < 0 || nx < 1 || ny < 1 || p_begin < 0 || p_count < 0 || p_begin > np || p_count > np - p_begin)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_coulomb: bad sizes or shard");
+    if (!std::isfinite(z) || !std::isfinite(h) || !(h > 0.f))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_coulomb: z must be finite and h finite and > 0");
+    if (p_count == 0) return LIME_OK;
+    if ((n_atoms > 0 && !atoms) || !V || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_coulomb: null pointer");
+    if ((n_atoms > 0 && !aligned16(atoms)) || (reinterpret_cast<uintptr_t>(V) & 3u) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_coulomb: atoms/ws 16-B, V 4-B aligned");
+    if (overlap(V, p_count * 4, atoms, n_atoms * 16) || overlap(ws, ws_bytes, atoms, n_atoms * 16) ||
+        overlap(ws, ws_bytes, V, p_count * 4))
+        return fail(LIME_ERR_ALIASING, "lime_map_coulomb: output/workspace overlap");
+    LIME_TRY(check_device());
+    if (ws_bytes < parboil::cp_workspace_bytes(n_atoms, p_count))
+        return fail(LIME_ERR_WORKSPACE, "lime_map_coulomb: workspace too small");
+    return launched(parboil::launch_cp(reinterpret_cast<const float4*>(atoms), n_atoms, nx, p_begin, p_count, z, h, V,
+                                       ws, static_cast<cudaStream_t>(stream)),
+                    "lime_map_coulomb");
+}
+
+size_t lime_map_mriq_workspace_bytes(int64_t n_k, int64_t x_count) {
+    if (n_k < 0 || x_count < 0) return 0;
+    return parboil::mriq_workspace_bytes(n_k, x_count);
+}
+
+lime_status lime_map_mriq(const float* kspace, int64_t n_k, const float* voxels, int64_t n_x, int64_t x_begin,
+                          int64_t x_count, float* Q, void* ws, size_t ws_bytes, void* stream) {
+    if (n_k < 0 || n_x < 0 || x_begin < 0 || x_count < 0 || x_begin > n_x || x_count > n_x - x_begin)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_mriq: bad sizes or shard");
+    if (x_count == 0) return LIME_OK;
+    if ((n_k > 0 && !kspace) || !voxels || !Q || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_mriq: null pointer");
+    if ((reinterpret_cast<uintptr_t>(kspace) & 3u) || (reinterpret_cast<uintptr_t>(voxels) & 3u) ||
+        (reinterpret_cast<uintptr_t>(Q) & 7u) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_mriq: kspace/voxels 4-B, Q 8-B, ws 16-B aligned");
+    const size_t qb = static_cast<size_t>(x_count) * 8;
+    if (overlap(Q, qb, kspace, n_k * 20) || overlap(Q, qb, voxels, n_x * 12) || overlap(ws, ws_bytes, kspace, n_k * 20) ||
+        overlap(ws, ws_bytes, voxels, n_x * 12) || overlap(ws, ws_bytes, Q, qb))
+        return fail(LIME_ERR_ALIASING, "lime_map_mriq: output/workspace overlap");
+    LIME_TRY(check_device());
+    if (ws_bytes < parboil::mriq_workspace_bytes(n_k, x_count))
+        return fail(LIME_ERR_WORKSPACE, "lime_map_mriq: workspace too small");
+    return launched(parboil::launch_mriq(kspace, n_k, voxels, x_begin, x_count, Q, ws, static_cast<cudaStream_t>(stream)),
+                    "lime_map_mriq");
+}
+
 // ============================================================================== Matmul
 lime_status lime_map_matmul_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
                                  void* stream) {

@@ -45,6 +45,16 @@ cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t
                    void* ws, cudaStream_t stream);
 }  // namespace mandel
 
+// ------------------------------------------------------------- Parboil CP / MRI-Q (F2)
+namespace parboil {
+size_t cp_workspace_bytes(int64_t n_atoms, int64_t points);
+size_t mriq_workspace_bytes(int64_t n_k, int64_t n_x);
+cudaError_t launch_cp(const float4* atoms, int64_t n_atoms, int32_t nx, int64_t p_begin, int64_t p_count, float z,
+                      float h, float* out, void* ws, cudaStream_t stream);
+cudaError_t launch_mriq(const float* kspace, int64_t n_k, const float* voxels, int64_t x_begin, int64_t x_count,
+                        float* out, void* ws, cudaStream_t stream);
+}  // namespace parboil
+
 // ------------------------------------------------------------------ Matmul
 namespace gemm {
 cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N,

@@ -3,7 +3,7 @@
     ncu --set full --clock-control none --import-source on -k regex:<kernel> -s 1 -c 1 \
         -o gpurun_out/prof_<which> python tools/prof_kernels.py <which>
 
-which: nbody1m | nbody1m_p8 | nbody4096 | bs_map | bs_fused | mandel | matmul | reduce
+which: nbody1m | nbody1m_p8 | nbody4096 | bs_map | bs_fused | mandel | matmul | reduce | cp | mriq
 """
 import os
 import sys
@@ -43,6 +43,15 @@ def main(which: str, reps: int = 3):
         B = torch.from_numpy(inputs.bf16_uniform(M, M, 4, 1).view(np.int16)).cuda().view(torch.bfloat16)
         for _ in range(reps):
             lime.map_matmul_bf16(A, B)
+    elif which == "cp":
+        atoms = torch.from_numpy(inputs.cp_atoms()).cuda()
+        for _ in range(reps):
+            lime.map_coulomb(atoms, inputs.CP_NX, inputs.CP_NY, inputs.CP_Z, inputs.CP_H)
+    elif which == "mriq":
+        k = torch.from_numpy(inputs.mriq_kspace()).cuda()
+        vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
+        for _ in range(reps):
+            lime.map_mriq(k, vx)
     elif which == "reduce":
         x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
         for _ in range(reps):

@@ -47,6 +47,14 @@ def main(which):
         b = torch.from_numpy(inputs.nbody_bodies(n, seed=1)).cuda()
         acc = torch.empty_like(b)
         out["nbody4096_us"] = 1e3 * time_launches(lambda: lime.map_nbody(b, 1e-4, out=acc), 50, 5, flush)[0]
+    if "parboil" in which:
+        atoms = torch.from_numpy(inputs.cp_atoms()).cuda()
+        V = torch.empty(inputs.CP_NX * inputs.CP_NY, device="cuda")
+        out["cp_us"] = 1e3 * time_launches(lambda: lime.map_coulomb(atoms, inputs.CP_NX, inputs.CP_NY, inputs.CP_Z, inputs.CP_H, out=V), 30, 3, flush)[0]
+        k = torch.from_numpy(inputs.mriq_kspace()).cuda()
+        vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
+        Q = torch.empty((vx.shape[0], 2), device="cuda")
+        out["mriq_us"] = 1e3 * time_launches(lambda: lime.map_mriq(k, vx, out=Q), 30, 3, flush)[0]
     if "reduce" in which:
         x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
         r = torch.empty((), dtype=torch.float32, device="cuda")
