@@ -348,6 +348,20 @@ def run_extras(peaks, flush):
     except lime.LimeError as e:
         out["matmul"] = {"workload": "configs[3]", "unavailable": str(e)}
 
+    # F3: double-precision N-Body (Table 3) at the config-5 per-GPU shape of P = 8; FP64-pipe
+    # bound: 16 FP64 ops per interaction at 64 lanes/clk/SM (microbench: 58.9 measured)
+    b64 = torch.from_numpy(inputs.nbody_bodies(1 << 20, seed=5).astype(np.float64)).cuda()
+    acc64 = torch.empty((1 << 17, 4), dtype=torch.float64, device="cuda")
+    med, _ = time_launches(lambda: lime.map_nbody_f64(b64, EPS2, 0, 1 << 17, out=acc64), 3, 1, flush)
+    inter = float(1 << 20) * (1 << 17)
+    fp64_peak = 64.0 * SMS_B200 * SM_MAX_MHZ_NOMINAL * 1e6
+    out["nbody_f64"] = {"workload": "F3: N-body fp64, 2^17 targets x 2^20 sources (config-5 shard at P=8)",
+                        "value": inter / (med * 1e-3), "unit": "interactions/s", "ms_per_launch": med,
+                        "roofline": {"bound": "alu", "achieved": 16 * inter / (med * 1e-3) / 1e12,
+                                     "peak": fp64_peak / 1e12, "unit": "T FP64 lane-ops/s",
+                                     "frac": 16 * inter / (med * 1e-3) / fp64_peak, "traffic": ncu_traffic("nbody_f64")}}
+    del b64, acc64
+
     # F2: Parboil-CP and MRI-Q at the paper's Table 3 sizes (L353-354); both are
     # bound by the MUFU (XU) pipe: 1 rsqrt (CP) / 1 sin + 1 cos (MRI-Q) per interaction.
     mufu_peak = 16.0 * SMS_B200 * SM_MAX_MHZ_NOMINAL * 1e6      # 16 lanes/clk/SM (microbench: 16.00)

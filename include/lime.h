@@ -116,6 +116,18 @@ lime_status lime_map_nbody(const float *bodies, int64_t n_src, int64_t tgt_begin
                            int64_t tgt_count, float eps2, float *accel,
                            void *ws, size_t ws_bytes, void *stream);
 
+/* Double-precision N-Body force map (Table 3 "N-Body
+ * ... Float / Double", L319-323, L372-373): the same map on bodies
+ * [n_src][4] double (x, y, z, m) -> accel [tgt_count][4] double (ax, ay, az, 0),
+ * eps2 finite and >= DBL_MIN; pointers 16-B aligned; same shard rules and the
+ * same split summation order as lime_map_nbody. The inverse square root is the
+ * MUFU approximation refined to full double precision.
+ * ws: lime_map_nbody_f64_workspace_bytes(n_src, tgt_count) bytes, zeroed once. */
+size_t lime_map_nbody_f64_workspace_bytes(int64_t n_src, int64_t tgt_count);
+lime_status lime_map_nbody_f64(const double *bodies, int64_t n_src, int64_t tgt_begin,
+                               int64_t tgt_count, double eps2, double *accel,
+                               void *ws, size_t ws_bytes, void *stream);
+
 /* N-Body integrator (the `forceAccumulator` sink, L112-114; R4):
  * semi-implicit Euler on n bodies, in place:
  *   vel.xyz += accel.xyz * dt ;  pos.xyz += vel.xyz * dt ;  pos.w (mass), vel.w kept.

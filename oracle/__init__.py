@@ -58,6 +58,7 @@ def _declare(L):
         "oracle_abi_version": (C.c_int, []),
         "oracle_nbody_accel": (None, [_p, _i64, _i64, _i64, _f, _p, _p]),
         "oracle_nbody_integrate": (None, [_p, _p, _p, _i64, _f, _p, _p]),
+        "oracle_nbody_accel_f64": (None, [_p, _i64, _i64, _i64, _d, _p, _p]),
         "oracle_normal_cdf": (_d, [_d]),
         "oracle_blackscholes": (None, [_p, _p, _p, _i64, _f, _f, _p, _p]),
         "oracle_blackscholes_sums": (None, [_p, _p, _p, _i64, _f, _f, _p]),
@@ -108,6 +109,19 @@ def nbody_accel(bodies, eps2: float, tgt_begin: int = 0, tgt_count: int | None =
     acc = np.zeros((tgt_count, 3), dtype=np.float64)
     mag = np.zeros(tgt_count, dtype=np.float64) if with_mag else None
     lib().oracle_nbody_accel(_ptr(b), n, tgt_begin, tgt_count, float(eps2), _ptr(acc), _ptr(mag))
+    return (acc, mag) if with_mag else acc
+
+
+def nbody_accel_f64(bodies, eps2: float, tgt_begin: int = 0, tgt_count: int | None = None,
+                    with_mag: bool = False):
+    """oracle_nbody_accel_f64: double bodies [n][4] -> a_i double [count][3] (optionally A_i)."""
+    b = _c(bodies, np.float64).reshape(-1, 4)
+    n = b.shape[0]
+    if tgt_count is None:
+        tgt_count = n - tgt_begin
+    acc = np.zeros((tgt_count, 3), dtype=np.float64)
+    mag = np.zeros(tgt_count, dtype=np.float64) if with_mag else None
+    lib().oracle_nbody_accel_f64(_ptr(b), n, tgt_begin, tgt_count, float(eps2), _ptr(acc), _ptr(mag))
     return (acc, mag) if with_mag else acc
 
 

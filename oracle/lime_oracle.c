@@ -455,3 +455,35 @@ void oracle_mriq(const float *kspace, int64_t n_k, const float *voxels, int64_t 
         if (mag) mag[i] = m;
     }
 }
+
+/* ------------------------------------------------------------------------
+ * N-Body, double precision (Table 3: "N-Body ... 64KB / 128KB
+ * 48KB / 128KB Float / Double"; L319-323 single- and double-precision variants;
+ * SURVEY.md §8(f) F3). Same definition as oracle_nbody_accel (R1-R3) on fp64
+ * bodies [n][4] (x, y, z, m); accel [count][3] double; mag optional. */
+void oracle_nbody_accel_f64(const double *bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,
+                            double eps2, double *accel, double *mag)
+{
+    oracle_fp_env();
+    for (int64_t t = 0; t < tgt_count; ++t) {
+        const int64_t i = tgt_begin + t;
+        const double xi = bodies[4 * i + 0], yi = bodies[4 * i + 1], zi = bodies[4 * i + 2];
+        double ax = 0.0, ay = 0.0, az = 0.0, am = 0.0;
+        for (int64_t j = 0; j < n_src; ++j) {
+            const double dx = bodies[4 * j + 0] - xi;
+            const double dy = bodies[4 * j + 1] - yi;
+            const double dz = bodies[4 * j + 2] - zi;
+            const double d2 = dx * dx + dy * dy + dz * dz;
+            const double r2 = d2 + eps2;
+            const double s = bodies[4 * j + 3] / (r2 * sqrt(r2));
+            ax += s * dx;
+            ay += s * dy;
+            az += s * dz;
+            am += s * sqrt(d2);
+        }
+        accel[3 * t + 0] = ax;
+        accel[3 * t + 1] = ay;
+        accel[3 * t + 2] = az;
+        if (mag) mag[t] = am;
+    }
+}

@@ -52,6 +52,8 @@ SIGNATURES = {
     "lime_nbody_splits": (_int, [_i64]),
     "lime_map_nbody": (_int, [_p, _i64, _i64, _i64, _f, _p, _p, _sz, _p]),
     "lime_map_nbody_integrate": (_int, [_p, _p, _p, _i64, _f, _p]),
+    "lime_map_nbody_f64_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_map_nbody_f64": (_int, [_p, _i64, _i64, _i64, C.c_double, _p, _p, _sz, _p]),
     "lime_nbody_simulate_host_workspace_bytes": (_sz, [_i64]),
     "lime_nbody_simulate_host": (_int, [_p, _p, _i64, _i32, _f, _f, _p, _sz, _p]),
     "lime_map_blackscholes": (_int, [_p, _p, _p, _i64, _f, _f, _p, _p, _p]),
@@ -172,6 +174,23 @@ def map_nbody(bodies: torch.Tensor, eps2: float, tgt_begin: int = 0, tgt_count: 
     ws = workspace(bodies.device, "nbody", nbytes)
     _check(L.lime_map_nbody(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
                             ws.data_ptr(), ws.numel(), _stream(bodies.device)), "lime_map_nbody")
+    return out
+
+
+def map_nbody_f64(bodies: torch.Tensor, eps2: float, tgt_begin: int = 0, tgt_count: int | None = None,
+                  out: torch.Tensor | None = None) -> torch.Tensor:
+    """Double-precision N-Body map (F3): bodies [n][4] float64 -> accel [count][4] float64."""
+    L = load()
+    _dev_tensor(bodies, torch.float64, "bodies", 4)
+    n = bodies.shape[0]
+    if tgt_count is None:
+        tgt_count = n - tgt_begin
+    if out is None:
+        out = torch.empty((max(tgt_count, 0), 4), dtype=torch.float64, device=bodies.device)
+    _dev_tensor(out, torch.float64, "out", 4)
+    ws = workspace(bodies.device, "nbody64", L.lime_map_nbody_f64_workspace_bytes(n, max(tgt_count, 0)))
+    _check(L.lime_map_nbody_f64(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
+                                ws.data_ptr(), ws.numel(), _stream(bodies.device)), "lime_map_nbody_f64")
     return out
 
 

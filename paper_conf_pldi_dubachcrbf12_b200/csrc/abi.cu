@@ -164,6 +164,32 @@ lime_status lime_map_nbody(const float* bodies, int64_t n_src, int64_t tgt_begin
                     "lime_map_nbody");
 }
 
+size_t lime_map_nbody_f64_workspace_bytes(int64_t n_src, int64_t tgt_count) {
+    if (n_src < 0 || tgt_count < 0) return 0;
+    return nbody64::workspace_bytes(n_src, tgt_count);
+}
+
+lime_status lime_map_nbody_f64(const double* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count, double eps2,
+                               double* accel, void* ws, size_t ws_bytes, void* stream) {
+    if (n_src < 0 || tgt_begin < 0 || tgt_count < 0 || tgt_begin > n_src || tgt_count > n_src - tgt_begin)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_f64: shard outside [0, n_src)");
+    if (!(std::isfinite(eps2) && eps2 >= 2.2250738585072014e-308))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_f64: eps2 must be finite and >= DBL_MIN");
+    if (tgt_count == 0) return LIME_OK;
+    if (!bodies || !accel || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_f64: null pointer");
+    if (!aligned16(bodies) || !aligned16(accel) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_nbody_f64: bodies, accel and ws must be 16-byte aligned");
+    if (overlap(accel, tgt_count * 32, bodies, n_src * 32) || overlap(ws, ws_bytes, bodies, n_src * 32) ||
+        overlap(ws, ws_bytes, accel, tgt_count * 32))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody_f64: output/workspace overlap");
+    LIME_TRY(check_device());
+    if (ws_bytes < nbody64::workspace_bytes(n_src, tgt_count))
+        return fail(LIME_ERR_WORKSPACE, "lime_map_nbody_f64: workspace too small");
+    return launched(nbody64::launch_force(bodies, n_src, tgt_begin, tgt_count, eps2, accel, ws,
+                                          static_cast<cudaStream_t>(stream)),
+                    "lime_map_nbody_f64");
+}
+
 lime_status lime_map_nbody_integrate(float* pos, float* vel, const float* accel, int64_t n, float dt, void* stream) {
     if (n < 0) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_integrate: n < 0");
     if (!std::isfinite(dt)) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_integrate: dt not finite");

@@ -29,6 +29,12 @@ cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int6
                              cudaStream_t stream);
 }  // namespace nbody
 
+namespace nbody64 {   // F3: double precision
+size_t workspace_bytes(int64_t n_src, int64_t tgt_count);
+cudaError_t launch_force(const double* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count, double eps2,
+                         double* accel, void* ws, cudaStream_t stream);
+}  // namespace nbody64
+
 // ----------------------------------------------------------- Black-Scholes
 namespace bs {
 cudaError_t launch_map(const float* S, const float* X, const float* T, int64_t n, float r,

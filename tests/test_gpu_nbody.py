@@ -134,3 +134,31 @@ def test_staging_ablation_variants_bit_identical(lime, n, count):
         with lime.nbody_variant(v):
             got = lime.map_nbody(b, float(EPS2), 0, count).cpu()
         assert torch.equal(got, ref), v
+
+
+# ------------------------------------------------------- F3: double precision (Table 3)
+NBODY64_RTOL = 1e-12   # fp64 with reordered summation
+
+
+@pytest.mark.parametrize("n", [1, 2, 33, 1000, 4096, 5000])
+def test_nbody_f64_matches_oracle(lime, n):
+    b = inputs.nbody_bodies(n, seed=40 + n).astype(np.float64)
+    b[:, :3] += 1e-9 * (inputs.uniform24(n, 5, 3 * n).reshape(n, 3) - 0.5)     # use the fp64 mantissa
+    acc = lime.map_nbody_f64(_dev(b), 1e-4).cpu().numpy()
+    ref, mag = oracle.nbody_accel_f64(b, 1e-4, with_mag=True)
+    assert nbody_rel_err(acc, ref, mag).max() <= NBODY64_RTOL
+    assert np.all(acc[:, 3] == 0.0)
+
+
+def test_nbody_f64_shards_and_config5_sample(lime):
+    n = 1 << 16
+    b = inputs.nbody_bodies(n, seed=44).astype(np.float64)
+    bd = _dev(b)
+    full = lime.map_nbody_f64(bd, 1e-4).cpu()
+    for P in (2, 8):
+        parts = [lime.map_nbody_f64(bd, 1e-4, r * n // P, n // P).cpu() for r in range(P)]
+        assert torch.equal(torch.cat(parts), full)
+    rows = np.random.default_rng(1).choice(n, 64, replace=False)
+    ref = np.stack([oracle.nbody_accel_f64(b, 1e-4, int(r), 1, with_mag=True)[0][0] for r in rows])
+    mag = np.array([oracle.nbody_accel_f64(b, 1e-4, int(r), 1, with_mag=True)[1][0] for r in rows])
+    assert nbody_rel_err(full.numpy()[rows], ref, mag).max() <= NBODY64_RTOL

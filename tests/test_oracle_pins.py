@@ -451,3 +451,19 @@ def test_mriq_shift_theorem_and_brute_force():
     pm = a[:, 3] ** 2 + a[:, 4] ** 2
     np.testing.assert_allclose(Q[:, 0], (pm * np.cos(arg)).sum(1), rtol=1e-11, atol=1e-11)
     np.testing.assert_allclose(Q[:, 1], (pm * np.sin(arg)).sum(1), rtol=1e-11, atol=1e-11)
+
+
+# =========================================== N-Body fp64 (F3, Table 3)
+
+def test_nbody_f64_matches_pins_and_fp32_oracle():
+    # Newton far field and attraction in double; agrees with the fp32-input oracle on fp32 data
+    b = np.array([[0, 0, 0, 0.125], [0, 2.0, 0, 0.25]], dtype=np.float64)
+    a = oracle.nbody_accel_f64(b, 1e-14)
+    assert a[0, 1] > 0 and abs(a[0, 1] - 0.25 / 4.0) <= 1e-12
+    b32 = inputs.nbody_bodies(200, seed=3)
+    np.testing.assert_array_equal(oracle.nbody_accel_f64(b32.astype(np.float64), float(np.float32(1e-4))),
+                                  oracle.nbody_accel(b32, np.float32(1e-4)))
+    bd = inputs.nbody_bodies(300, seed=4).astype(np.float64) + 1e-9 * inputs.uniform24(4, 9, 1200).reshape(300, 4)
+    acc, A = oracle.nbody_accel_f64(bd, 1e-4, with_mag=True)
+    m = bd[:, 3]
+    assert np.linalg.norm((m[:, None] * acc).sum(0)) <= 1e-14 * (m * A).sum()

@@ -47,6 +47,13 @@ def main(which):
         b = torch.from_numpy(inputs.nbody_bodies(n, seed=1)).cuda()
         acc = torch.empty_like(b)
         out["nbody4096_us"] = 1e3 * time_launches(lambda: lime.map_nbody(b, 1e-4, out=acc), 50, 5, flush)[0]
+    if "nbody64" in which:
+        for n, cnt in ((4096, 4096), (1 << 20, 1 << 17)):
+            b = torch.from_numpy(inputs.nbody_bodies(n, seed=1).astype(np.float64)).cuda()
+            acc = torch.empty((cnt, 4), dtype=torch.float64, device="cuda")
+            ms = time_launches(lambda: lime.map_nbody_f64(b, 1e-4, 0, cnt, out=acc), 5 if n > 4096 else 30, 2, flush)[0]
+            out[f"nbody64_{n}x{cnt}_ms"] = ms
+            out[f"nbody64_{n}x{cnt}_Gint_s"] = n * cnt / ms / 1e6
     if "parboil" in which:
         atoms = torch.from_numpy(inputs.cp_atoms()).cuda()
         V = torch.empty(inputs.CP_NX * inputs.CP_NY, device="cuda")
