@@ -68,6 +68,9 @@ def _declare(L):
         "oracle_matmul_bf16_entries": (None, [_p, _p, _i64, _p, _p, _i64, _p, _p]),
         "oracle_coulomb_potential": (None, [_p, _i64, _i32, _i32, _i32, _f, _f, _p, _p]),
         "oracle_mriq": (None, [_p, _i64, _p, _i64, _p, _p]),
+        "oracle_series": (None, [_i64, _i64, _i32, _p, _p]),
+        "oracle_idea_keys": (None, [_p, _p, _p]),
+        "oracle_idea": (None, [_p, _p, _i64, _p]),
         "oracle_reduce_sum_f32": (_d, [_p, _i64]),
         "oracle_reduce_sum_f64": (_d, [_p, _i64]),
         "oracle_reduce_sum_i32": (_i32, [_p, _i64]),
@@ -267,6 +270,39 @@ def mriq(kspace, voxels, threads: int = 1):
 
     _parallel(work, vx.shape[0], threads)
     return out, mag
+
+
+# ----------------------------------------------------------- JG-Series / JG-Crypt (F4)
+def series(n0: int, count: int, m: int = 1000, threads: int = 1):
+    """oracle_series: (a_n, b_n) double [count][2] and the bound T[|f|] [count]."""
+    out = np.zeros((count, 2), dtype=np.float64)
+    mag = np.zeros(count, dtype=np.float64)
+    L = lib()
+
+    def work(lo, hi):
+        if hi > lo:
+            L.oracle_series(n0 + lo, hi - lo, m, out[lo:hi].ctypes.data, mag[lo:hi].ctypes.data)
+
+    _parallel(work, count, threads)
+    return out, mag
+
+
+def idea_keys(key):
+    """oracle_idea_keys: (encryption, decryption) sub-keys, uint16 [52] each."""
+    k = _c(key, np.uint16)
+    ek = np.zeros(52, dtype=np.uint16)
+    dk = np.zeros(52, dtype=np.uint16)
+    lib().oracle_idea_keys(_ptr(k), _ptr(ek), _ptr(dk))
+    return ek, dk
+
+
+def idea(data, subkeys):
+    """oracle_idea: IDEA-ECB of a byte array (len % 8 == 0) with the given 52 sub-keys."""
+    d = _c(data, np.uint8)
+    z = _c(subkeys, np.uint16)
+    out = np.zeros_like(d)
+    lib().oracle_idea(_ptr(d), _ptr(out), d.shape[0], _ptr(z))
+    return out
 
 
 # ------------------------------------------------------------- Reductions

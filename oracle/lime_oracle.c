@@ -487,3 +487,148 @@ void oracle_nbody_accel_f64(const double *bodies, int64_t n_src, int64_t tgt_beg
         if (mag) mag[t] = am;
     }
 }
+
+/* ------------------------------------------------------------------------
+ * JG-Series: Fourier coefficient analysis (Table 3 "JG-Series
+ * Fourier coefficient analysis 780KB / 1560KB Float / Double"; SURVEY.md §8(f)
+ * F4). The paper ports the Java Grande Forum "Series" kernel; reading
+ * DESIGN.md R14 follows that kernel step by step: the first N coefficient
+ * pairs of f(x) = (x+1)^x on [0, 2] with omega = pi,
+ *   a_0 = T(0, 0) / 2, b_0 = 0 ;  a_n = T(n pi, cos), b_n = T(n pi, sin) (n >= 1)
+ * where T is JGF's TrapezoidIntegrate(0, 2, m, omega_n, select):
+ *   dx = 2/m; r = g(0)/2; for i = 1 .. m-2: r += g(x_i); r = (r + g(2)/2) dx
+ * -- JGF's loop `--nsteps; while (--nsteps > 0)` visits the interior nodes
+ * x_1 .. x_{m-2} only (node x_{m-1} is skipped), and that is kept. Nodes are
+ * x_i = i dx (one rounding; JGF accumulates x += dx, a < 1e-12 difference).
+ * g(x) = f(x) [select 0], f(x) cos(omega x) [1], f(x) sin(omega x) [2].
+ * In double. out[k][2] = (a_n, b_n) for n = n0 + k; mag[k] = T over |f|. */
+static double series_g(double x, double omegan, int select)
+{
+    const double f = pow(x + 1.0, x);
+    if (select == 0) return f;
+    return select == 1 ? f * cos(omegan * x) : f * sin(omegan * x);
+}
+
+static double series_trapezoid(double x0, double x1, int32_t nsteps, double omegan, int select)
+{
+    const double dx = (x1 - x0) / nsteps;
+    double r = series_g(x0, omegan, select) / 2.0;
+    if (nsteps != 1)
+        for (int32_t i = 1; i < nsteps - 1; ++i) r += series_g(x0 + i * dx, omegan, select);
+    return (r + series_g(x1, omegan, select) / 2.0) * dx;
+}
+
+void oracle_series(int64_t n0, int64_t count, int32_t m, double *out, double *mag)
+{
+    oracle_fp_env();
+    const double omega = 3.1415926535897932;
+    for (int64_t k = 0; k < count; ++k) {
+        const int64_t n = n0 + k;
+        if (n == 0) {
+            out[2 * k + 0] = series_trapezoid(0.0, 2.0, m, 0.0, 0) / 2.0;
+            out[2 * k + 1] = 0.0;
+        } else {
+            out[2 * k + 0] = series_trapezoid(0.0, 2.0, m, omega * (double)n, 1);
+            out[2 * k + 1] = series_trapezoid(0.0, 2.0, m, omega * (double)n, 2);
+        }
+        if (mag) mag[k] = series_trapezoid(0.0, 2.0, m, 0.0, 0);    /* f > 0: T[|f|] = T[f] */
+    }
+}
+
+/* ------------------------------------------------------------------------
+ * JG-Crypt: IDEA block cipher over a byte array (Table 3
+ * "JG-Crypt IDEA encryption 3MB 3MB Byte"). Reading
+ * DESIGN.md R15: IDEA (Lai & Massey 1991) in ECB mode, 8-byte blocks of four
+ * big-endian 16-bit words, 8 rounds + output transform, 52 sub-keys from the
+ * 128-bit key (25-bit rotations); decryption uses the inverted sub-keys. The
+ * byte array length must be a multiple of 8. */
+static uint16_t idea_mul(uint16_t a, uint16_t b)
+{
+    /* multiplication modulo 2^16 + 1, with 0 standing for 2^16 */
+    const uint32_t aa = a ? a : 65536u, bb = b ? b : 65536u;
+    const uint64_t p = ((uint64_t)aa * bb) % 65537u;
+    return (uint16_t)(p == 65536u ? 0 : p);
+}
+
+static uint16_t idea_mul_inv(uint16_t a)
+{
+    /* a^(65537-2) mod 65537 (Fermat), with 0 <-> 2^16 */
+    const uint64_t mod = 65537u;
+    uint64_t base = a ? a : 65536u, r = 1, e = mod - 2;
+    while (e) {
+        if (e & 1) r = (r * base) % mod;
+        base = (base * base) % mod;
+        e >>= 1;
+    }
+    return (uint16_t)(r == 65536u ? 0 : r);
+}
+
+void oracle_idea_keys(const uint16_t key[8], uint16_t ek[52], uint16_t dk[52])
+{
+    /* encryption sub-keys: the 128-bit key, then repeatedly rotated left by 25 bits */
+    uint8_t k[16];
+    for (int i = 0; i < 8; ++i) { k[2 * i] = (uint8_t)(key[i] >> 8); k[2 * i + 1] = (uint8_t)key[i]; }
+    for (int s = 0; s < 52; ++s) {
+        const int rot = 25 * (s / 8);               /* bits rotated so far */
+        const int w = s % 8;
+        uint16_t v = 0;
+        for (int b = 0; b < 16; ++b) {
+            const int bit = (16 * w + b + rot) % 128;   /* MSB-first bit index in k */
+            v = (uint16_t)((v << 1) | ((k[bit / 8] >> (7 - bit % 8)) & 1));
+        }
+        ek[s] = v;
+    }
+    /* decryption sub-keys */
+    dk[0] = idea_mul_inv(ek[48]);
+    dk[1] = (uint16_t)(0u - ek[49]);
+    dk[2] = (uint16_t)(0u - ek[50]);
+    dk[3] = idea_mul_inv(ek[51]);
+    for (int r = 1; r < 8; ++r) {
+        const int e = 48 - 6 * r, d = 6 * r;
+        dk[d - 2] = ek[e + 4];
+        dk[d - 1] = ek[e + 5];
+        dk[d + 0] = idea_mul_inv(ek[e + 0]);
+        dk[d + 1] = (uint16_t)(0u - ek[e + 2]);     /* middle rounds swap the two additive keys */
+        dk[d + 2] = (uint16_t)(0u - ek[e + 1]);
+        dk[d + 3] = idea_mul_inv(ek[e + 3]);
+    }
+    dk[46] = ek[4];
+    dk[47] = ek[5];
+    dk[48] = idea_mul_inv(ek[0]);
+    dk[49] = (uint16_t)(0u - ek[1]);
+    dk[50] = (uint16_t)(0u - ek[2]);
+    dk[51] = idea_mul_inv(ek[3]);
+}
+
+static void idea_block(const uint8_t in[8], uint8_t out[8], const uint16_t z[52])
+{
+    uint16_t x1 = (uint16_t)(in[0] << 8 | in[1]), x2 = (uint16_t)(in[2] << 8 | in[3]);
+    uint16_t x3 = (uint16_t)(in[4] << 8 | in[5]), x4 = (uint16_t)(in[6] << 8 | in[7]);
+    for (int r = 0; r < 8; ++r) {
+        const uint16_t *k = z + 6 * r;
+        x1 = idea_mul(x1, k[0]);
+        x2 = (uint16_t)(x2 + k[1]);
+        x3 = (uint16_t)(x3 + k[2]);
+        x4 = idea_mul(x4, k[3]);
+        const uint16_t t0 = idea_mul((uint16_t)(x1 ^ x3), k[4]);
+        const uint16_t t1 = idea_mul((uint16_t)(t0 + (x2 ^ x4)), k[5]);
+        const uint16_t t2 = (uint16_t)(t0 + t1);
+        x1 ^= t1;
+        x4 ^= t2;
+        const uint16_t a = (uint16_t)(x2 ^ t2);
+        x2 = (uint16_t)(x3 ^ t1);
+        x3 = a;
+    }
+    const uint16_t y1 = idea_mul(x1, z[48]);
+    const uint16_t y2 = (uint16_t)(x3 + z[49]);      /* undo the last round's swap */
+    const uint16_t y3 = (uint16_t)(x2 + z[50]);
+    const uint16_t y4 = idea_mul(x4, z[51]);
+    out[0] = (uint8_t)(y1 >> 8); out[1] = (uint8_t)y1; out[2] = (uint8_t)(y2 >> 8); out[3] = (uint8_t)y2;
+    out[4] = (uint8_t)(y3 >> 8); out[5] = (uint8_t)y3; out[6] = (uint8_t)(y4 >> 8); out[7] = (uint8_t)y4;
+}
+
+/* ECB over nbytes (multiple of 8) with sub-keys z (ek to encrypt, dk to decrypt) */
+void oracle_idea(const uint8_t *in, uint8_t *out, int64_t nbytes, const uint16_t z[52])
+{
+    for (int64_t i = 0; i + 8 <= nbytes; i += 8) idea_block(in + i, out + i, z);
+}

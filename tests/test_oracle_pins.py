@@ -467,3 +467,42 @@ def test_nbody_f64_matches_pins_and_fp32_oracle():
     acc, A = oracle.nbody_accel_f64(bd, 1e-4, with_mag=True)
     m = bd[:, 3]
     assert np.linalg.norm((m[:, None] * acc).sum(0)) <= 1e-14 * (m * A).sum()
+
+
+# ============================================ JG-Series / JG-Crypt (F4, Table 3)
+
+def test_series_matches_jgf_reference_values():
+    g = _golden("jgf_series_ref.json")
+    out, _ = oracle.series(0, 4)
+    np.testing.assert_allclose(out, np.array(g["ref"]), rtol=0, atol=1e-11)
+
+
+def test_series_integral_and_bounds():
+    # a_0 = (1/2) [int_0^2 (x+1)^x dx - dx f(x_999)] up to the trapezoid error O(dx^2): the exact
+    # integral (scipy quad, independent) minus JGF's skipped node x_999 = 1.998.
+    from scipy.integrate import quad
+    I, _ = quad(lambda x: (x + 1.0) ** x, 0.0, 2.0, epsabs=1e-13)
+    skipped = 0.002 * (1.998 + 1.0) ** 1.998
+    out, mag = oracle.series(0, 200)
+    assert abs(out[0, 0] - (I - skipped) / 2) < 1e-5 and out[0, 1] == 0.0
+    assert np.all(np.abs(out) <= mag[:, None] * (1 + 1e-12))
+    # coefficients of a smooth non-periodic function decay like 1/n: |b_n| n stays bounded
+    n = np.arange(1, 200)
+    assert np.abs(out[1:, 1] * n).max() < 20
+
+
+def test_idea_published_test_vector_and_inverse():
+    g = _golden("idea_test_vector.json")
+    ek, dk = oracle.idea_keys(g["key"])
+    pt = np.array(g["plaintext_bytes"], dtype=np.uint8)
+    ct = oracle.idea(pt, ek)
+    assert ct.tolist() == g["ciphertext_bytes"]
+    assert oracle.idea(ct, dk).tolist() == pt.tolist()
+    data = (inputs.splitmix64(3, 0, 4096) & np.uint64(0xFF)).astype(np.uint8)
+    ek2, dk2 = oracle.idea_keys([0x2BD6, 0x459F, 0x82C5, 0xB300, 0x952C, 0x4910, 0x4881, 0xFF48])
+    enc = oracle.idea(data, ek2)
+    assert not np.array_equal(enc, data) and np.array_equal(oracle.idea(enc, dk2), data)
+    # ECB: equal plaintext blocks give equal ciphertext blocks
+    rep = np.tile(data[:8], 4)
+    e = oracle.idea(rep, ek2).reshape(4, 8)
+    assert all(np.array_equal(e[0], e[k]) for k in range(4))
