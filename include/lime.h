@@ -236,6 +236,36 @@ lime_status lime_map_mriq(const float *kspace, int64_t n_k, const float *voxels,
                           int64_t x_count, float *Q, void *ws, size_t ws_bytes, void *stream);
 
 /* ===========================================================================
+ * JG-Series (Table 3; definition DESIGN.md
+ * R14 = the Java Grande "Series" kernel incl. its trapezoid loop): coefficient
+ * pairs of f(x) = (x+1)^x on [0, 2], out[k] = (a_n, b_n) for n = n0 + k,
+ * k in [0, count): a_0 = T[f]/2, b_0 = 0, a_n = T[f cos(n pi x)],
+ * b_n = T[f sin(n pi x)], 1000-step trapezoid. out [count][2] float (f32) or
+ * double (f64), naturally aligned. Phases are reduced exactly in integers
+ * ((n i) mod 1000) before table lookup, so any n up to 2^40 is accurate.
+ * ws: lime_map_series_workspace_bytes() bytes (node and cos/sin tables).
+ * =========================================================================== */
+size_t lime_map_series_workspace_bytes(void);
+lime_status lime_map_series_f32(int64_t n0, int64_t count, float *out, void *ws, size_t ws_bytes,
+                                void *stream);
+lime_status lime_map_series_f64(int64_t n0, int64_t count, double *out, void *ws, size_t ws_bytes,
+                                void *stream);
+
+/* ===========================================================================
+ * JG-Crypt (Table 3; definition DESIGN.md
+ * R15): IDEA in ECB mode, a map over 8-byte blocks (four big-endian 16-bit
+ * words). lime_idea_key_schedule (HOST pointers, no device work) expands a
+ * 128-bit key key[8] into the 52 encryption sub-keys ek and decryption
+ * sub-keys dk. lime_map_idea enciphers nbytes (a multiple of 8) from `in` to
+ * `out` (device, 16-B aligned, no overlap) with the 52 sub-keys `subkeys`
+ * (HOST pointer; copied into the launch parameters): pass ek to encrypt, dk
+ * to decrypt. Bit-exact.
+ * =========================================================================== */
+void lime_idea_key_schedule(const uint16_t *key, uint16_t *ek, uint16_t *dk);
+lime_status lime_map_idea(const uint8_t *in, uint8_t *out, int64_t nbytes, const uint16_t *subkeys,
+                          void *stream);
+
+/* ===========================================================================
  * Reductions `!` over an array x[n] (L160-163; L188-189 "the compiler may
  * infer a parallel reduction"; R9). Tree: per-thread fold ->
  * warp shuffle -> CTA -> last CTA combines the CTA partials in index order.

@@ -64,6 +64,11 @@ SIGNATURES = {
     "lime_reduce_workspace_bytes": (_sz, []),
     "lime_map_coulomb_workspace_bytes": (_sz, [_i64, _i64]),
     "lime_map_coulomb": (_int, [_p, _i64, _i32, _i32, _i64, _i64, _f, _f, _p, _p, _sz, _p]),
+    "lime_map_series_workspace_bytes": (_sz, []),
+    "lime_map_series_f32": (_int, [_i64, _i64, _p, _p, _sz, _p]),
+    "lime_map_series_f64": (_int, [_i64, _i64, _p, _p, _sz, _p]),
+    "lime_idea_key_schedule": (None, [_p, _p, _p]),
+    "lime_map_idea": (_int, [_p, _p, _i64, _p, _p]),
     "lime_map_mriq_workspace_bytes": (_sz, [_i64, _i64]),
     "lime_map_mriq": (_int, [_p, _i64, _p, _i64, _i64, _i64, _p, _p, _sz, _p]),
 }
@@ -302,6 +307,42 @@ def map_mriq(kspace: torch.Tensor, voxels: torch.Tensor, x_begin: int = 0, x_cou
     ws = workspace(voxels.device, "mriq", L.lime_map_mriq_workspace_bytes(kspace.shape[0], max(x_count, 0)))
     _check(L.lime_map_mriq(kspace.data_ptr(), kspace.shape[0], voxels.data_ptr(), n_x, x_begin, x_count,
                            out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(voxels.device)), "lime_map_mriq")
+    return out
+
+
+# ------------------------------------------------------- JG-Series / JG-Crypt (F4)
+def map_series(n0: int, count: int, dtype=torch.float32, device="cuda", out=None) -> torch.Tensor:
+    """JG-Series coefficient pairs (a_n, b_n) for n in [n0, n0+count) -> [count][2]."""
+    L = load()
+    dev = torch.device(device)
+    out = torch.empty((count, 2), dtype=dtype, device=dev) if out is None else out
+    ws = workspace(dev, "series", L.lime_map_series_workspace_bytes())
+    fn = L.lime_map_series_f64 if dtype == torch.float64 else L.lime_map_series_f32
+    _check(fn(n0, count, out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_series")
+    return out
+
+
+def idea_key_schedule(key):
+    """IDEA sub-keys (ek, dk), each 52 uint16 words, from a 128-bit key given as 8 uint16 words."""
+    import numpy as np
+    k = np.ascontiguousarray(key, dtype=np.uint16)
+    if k.shape != (8,):
+        raise ValueError("key must be 8 16-bit words")
+    ek = np.zeros(52, dtype=np.uint16)
+    dk = np.zeros(52, dtype=np.uint16)
+    load().lime_idea_key_schedule(k.ctypes.data, ek.ctypes.data, dk.ctypes.data)
+    return ek, dk
+
+
+def map_idea(data: torch.Tensor, subkeys, out=None) -> torch.Tensor:
+    """IDEA-ECB of a uint8 CUDA tensor (length % 8 == 0) with 52 sub-keys (ek encrypts, dk decrypts)."""
+    import numpy as np
+    L = load()
+    _dev_tensor(data, torch.uint8, "data")
+    z = np.ascontiguousarray(subkeys, dtype=np.uint16)
+    out = torch.empty_like(data) if out is None else out
+    _check(L.lime_map_idea(data.data_ptr(), out.data_ptr(), data.numel(), z.ctypes.data, _stream(data.device)),
+           "lime_map_idea")
     return out
 
 

@@ -370,6 +370,50 @@ lime_status lime_map_mriq(const float* kspace, int64_t n_k, const float* voxels,
                     "lime_map_mriq");
 }
 
+// ========================================================================= JG-Series / JG-Crypt
+size_t lime_map_series_workspace_bytes(void) { return jgf::series_workspace_bytes(true); }
+
+static lime_status series_entry(const char* fn, int64_t n0, int64_t count, void* out, size_t esz, void* ws,
+                                size_t ws_bytes, void* stream) {
+    if (n0 < 0 || count < 0 || n0 > (1LL << 40) || count > (1LL << 40))
+        return fail(LIME_ERR_INVALID_ARG, "%s: n0, count must be in [0, 2^40]", fn);
+    if (count == 0) return LIME_OK;
+    if (!out || !ws) return fail(LIME_ERR_INVALID_ARG, "%s: null pointer", fn);
+    if ((reinterpret_cast<uintptr_t>(out) % esz) != 0 || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "%s: out needs natural alignment, ws 16-B", fn);
+    if (overlap(out, static_cast<size_t>(count) * 2 * esz, ws, ws_bytes))
+        return fail(LIME_ERR_ALIASING, "%s: out overlaps ws", fn);
+    LIME_TRY(check_device());
+    if (ws_bytes < jgf::series_workspace_bytes(esz == 8)) return fail(LIME_ERR_WORKSPACE, "%s: workspace too small", fn);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    return launched(esz == 8 ? jgf::launch_series_f64(n0, count, static_cast<double*>(out), ws, s)
+                             : jgf::launch_series_f32(n0, count, static_cast<float*>(out), ws, s),
+                    fn);
+}
+
+lime_status lime_map_series_f32(int64_t n0, int64_t count, float* out, void* ws, size_t ws_bytes, void* stream) {
+    return series_entry("lime_map_series_f32", n0, count, out, 4, ws, ws_bytes, stream);
+}
+
+lime_status lime_map_series_f64(int64_t n0, int64_t count, double* out, void* ws, size_t ws_bytes, void* stream) {
+    return series_entry("lime_map_series_f64", n0, count, out, 8, ws, ws_bytes, stream);
+}
+
+void lime_idea_key_schedule(const uint16_t* key, uint16_t* ek, uint16_t* dk) {
+    if (!key || !ek || !dk) return;
+    jgf::idea_key_schedule(key, ek, dk);
+}
+
+lime_status lime_map_idea(const uint8_t* in, uint8_t* out, int64_t nbytes, const uint16_t* subkeys, void* stream) {
+    if (nbytes < 0 || (nbytes % 8) != 0) return fail(LIME_ERR_INVALID_ARG, "lime_map_idea: nbytes must be a multiple of 8");
+    if (nbytes == 0) return LIME_OK;
+    if (!in || !out || !subkeys) return fail(LIME_ERR_INVALID_ARG, "lime_map_idea: null pointer");
+    if (!aligned16(in) || !aligned16(out)) return fail(LIME_ERR_MISALIGNED, "lime_map_idea: in/out must be 16-byte aligned");
+    if (overlap(in, nbytes, out, nbytes)) return fail(LIME_ERR_ALIASING, "lime_map_idea: out overlaps in");
+    LIME_TRY(check_device());
+    return launched(jgf::launch_idea(in, out, nbytes, subkeys, static_cast<cudaStream_t>(stream)), "lime_map_idea");
+}
+
 // ============================================================================== Matmul
 lime_status lime_map_matmul_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
                                  void* stream) {

@@ -61,6 +61,15 @@ cudaError_t launch_mriq(const float* kspace, int64_t n_k, const float* voxels, i
                         float* out, void* ws, cudaStream_t stream);
 }  // namespace parboil
 
+// ------------------------------------------------------------- JG-Series / JG-Crypt (F4)
+namespace jgf {
+size_t series_workspace_bytes(bool f64);
+cudaError_t launch_series_f32(int64_t n0, int64_t count, float* out, void* ws, cudaStream_t stream);
+cudaError_t launch_series_f64(int64_t n0, int64_t count, double* out, void* ws, cudaStream_t stream);
+void idea_key_schedule(const uint16_t key[8], uint16_t ek[52], uint16_t dk[52]);
+cudaError_t launch_idea(const uint8_t* in, uint8_t* out, int64_t nbytes, const uint16_t* subkeys, cudaStream_t stream);
+}  // namespace jgf
+
 // ------------------------------------------------------------------ Matmul
 namespace gemm {
 cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N,

@@ -170,3 +170,18 @@ def mriq_voxels(n: int = MRIQ_VOXELS, seed: int = 9) -> np.ndarray:
     for c in range(3):
         out[:, c] = (uniform24(seed, c, n).astype(np.float64) - 0.5).astype(np.float32)
     return out
+
+
+# ------------------------------------------------------- JG-Series / JG-Crypt
+SERIES_N = 100_000          # Table 3: 780 KB of fp32 (a_n, b_n) pairs (L355; JGF size B)
+CRYPT_BYTES = 3 << 20       # Table 3: 3 MB byte array (L354-355)
+
+
+def crypt_data(nbytes: int = CRYPT_BYTES, seed: int = 10) -> np.ndarray:
+    """nbytes uniform random bytes (uint8)."""
+    return _chunked(lambda o, m: (splitmix64(seed, 0, m, o) & np.uint64(0xFF)).astype(np.uint8), nbytes)
+
+
+def crypt_key(seed: int = 11) -> np.ndarray:
+    """A seeded 128-bit IDEA key as eight 16-bit words."""
+    return (splitmix64(seed, 0, 8) & np.uint64(0xFFFF)).astype(np.uint16)
