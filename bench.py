@@ -388,6 +388,30 @@ def run_extras(peaks, flush):
                                         "frac": 2 * inter / (med * 1e-3) / mufu_peak, "traffic": ncu_traffic("parboil_mriq")}}
     del atoms, V, k, vx, Q
 
+    # F4: JG-Series (100,000 coefficient pairs, Table 3) and JG-Crypt (IDEA over 3 MiB, L354-355)
+    for dt, nm in ((torch.float32, "jg_series_f32"), (torch.float64, "jg_series_f64")):
+        so = torch.empty((inputs.SERIES_N, 2), dtype=dt, device="cuda")
+        med, _ = time_launches(lambda: lime.map_series(0, inputs.SERIES_N, dtype=dt, out=so), 20, 3, flush)
+        terms = float(inputs.SERIES_N) * 1001
+        out[nm] = {"workload": f"F4: JG-Series {'fp32' if dt == torch.float32 else 'fp64'}, 100,000 coefficient pairs x 1001 nodes",
+                   "value": inputs.SERIES_N / (med * 1e-3), "unit": "coefficient pairs/s", "ms_per_launch": med,
+                   "terms_per_s": terms / (med * 1e-3),
+                   "roofline": {"bound": "smem", "achieved": terms * (16 if dt == torch.float32 else 32) / (med * 1e-3) / 1e9,
+                                "peak": 128.0 * SMS_B200 * SM_MAX_MHZ_NOMINAL * 1e6 / 1e9, "unit": "GB/s (shared-memory loads)",
+                                "frac": terms * (16 if dt == torch.float32 else 32) / (med * 1e-3) / (128.0 * SMS_B200 * SM_MAX_MHZ_NOMINAL * 1e6),
+                                "traffic": None}}
+        del so
+    data = torch.from_numpy(inputs.crypt_data()).cuda()
+    ek, _ = lime.idea_key_schedule(inputs.crypt_key())
+    enc = torch.empty_like(data)
+    med, _ = time_launches(lambda: lime.map_idea(data, ek, out=enc), 30, 3, flush)
+    gbs = 2.0 * data.numel() / (med * 1e-3) / 1e9
+    out["jg_crypt"] = {"workload": "F4: JG-Crypt IDEA-ECB over 3 MiB (Table 3)", "value": data.numel() / (med * 1e-3),
+                       "unit": "bytes/s", "ms_per_launch": med,
+                       "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
+                                    "traffic": None, "note": "3 MiB is latency-bound: one wave of 148 x 8 CTAs"}}
+    del data, enc
+
     # reduction `!`: sum over 2^28 fp32 (1 GiB)
     x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
     r = torch.empty((), dtype=torch.float32, device="cuda")
