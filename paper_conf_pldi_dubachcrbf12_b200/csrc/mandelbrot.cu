@@ -19,9 +19,9 @@
 namespace lime {
 namespace mandel {
 
-constexpr int kTileW = 16;   // pixels per warp tile row (8 lanes x 2 pixels)
-constexpr int kTileH = 4;    // rows per warp tile
-constexpr int kUnroll = 16;
+// A warp tile is (2 * LW) pixels wide and (32 / LW) rows tall (LW lanes per row, 2 pixels per
+// lane); the warp votes every UNROLL iterations. Variants are selected by the launch override
+// (per_thread = 1..5, see launch()); results never depend on them.
 
 struct Args {
     int32_t width, row_first, row_stride, row_count;
@@ -58,7 +58,9 @@ struct State {
     }
 };
 
+template <int LW, int UNROLL>
 __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Args a) {
+    constexpr int kTileW = 2 * LW, kTileH = 32 / LW;
     const unsigned lane = lane_id();
     for (;;) {
         int64_t tile = 0;
@@ -67,8 +69,8 @@ __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Arg
         if (tile >= a.ntiles) break;
         const int32_t tx = static_cast<int32_t>(tile % a.tiles_x);
         const int32_t ty = static_cast<int32_t>(tile / a.tiles_x);
-        const int32_t col = tx * kTileW + static_cast<int32_t>(lane & 7) * 2;
-        const int32_t k = ty * kTileH + static_cast<int32_t>(lane >> 3);
+        const int32_t col = tx * kTileW + static_cast<int32_t>(lane % LW) * 2;
+        const int32_t k = ty * kTileH + static_cast<int32_t>(lane / LW);
         const bool v0 = (col < a.width) && (k < a.row_count);
         const bool v1 = (col + 1 < a.width) && (k < a.row_count);
         const int32_t py = a.row_first + min(k, a.row_count - 1) * a.row_stride;
@@ -83,10 +85,10 @@ __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Arg
         st.a0 = st.a1 = true;
 
         int32_t it = 0;
-        while (it + kUnroll <= a.max_iter) {
+        while (it + UNROLL <= a.max_iter) {
 #pragma unroll
-            for (int u = 0; u < kUnroll; ++u) st.step();
-            it += kUnroll;
+            for (int u = 0; u < UNROLL; ++u) st.step();
+            it += UNROLL;
             if (!__any_sync(0xffffffffu, st.a0 || st.a1)) break;
         }
         if (__any_sync(0xffffffffu, st.a0 || st.a1)) {
@@ -106,6 +108,26 @@ __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Arg
     }
 }
 
+template <int LW, int UNROLL>
+static cudaError_t launch_t(Args& a, cudaStream_t stream) {
+    a.tiles_x = ceil_div<int32_t>(a.width, 2 * LW);
+    a.ntiles = static_cast<int64_t>(a.tiles_x) * ceil_div<int32_t>(a.row_count, 32 / LW);
+    int grid = launch_override().grid_ctas;
+    if (grid <= 0) {
+        static int per_sm = 0;
+        if (per_sm == 0) {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mandel_kernel<LW, UNROLL>, 256, 0);
+            if (per_sm <= 0) per_sm = 1;
+        }
+        grid = per_sm * device_num_sms();
+        const int64_t need = ceil_div<int64_t>(a.ntiles, 8);
+        if (need < grid) grid = static_cast<int>(need);
+    }
+    a.total_warps = static_cast<unsigned>(grid) * 8u;
+    mandel_kernel<LW, UNROLL><<<grid, 256, 0, stream>>>(a);
+    return cudaGetLastError();
+}
+
 cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t row_count, float x0,
                    float y0, float dx, float dy, int32_t max_iter, int32_t* counts, void* ws,
                    cudaStream_t stream) {
@@ -122,22 +144,16 @@ cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t
     a.max_iter = max_iter;
     a.counts = counts;
     a.queue = static_cast<unsigned*>(ws);
-    a.tiles_x = ceil_div<int32_t>(width, kTileW);
-    a.ntiles = static_cast<int64_t>(a.tiles_x) * ceil_div<int32_t>(row_count, kTileH);
-    int grid = launch_override().grid_ctas;
-    if (grid <= 0) {
-        static int per_sm = 0;
-        if (per_sm == 0) {
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mandel_kernel, 256, 0);
-            if (per_sm <= 0) per_sm = 1;
-        }
-        grid = per_sm * device_num_sms();
-        const int64_t need = ceil_div<int64_t>(a.ntiles, 8);
-        if (need < grid) grid = static_cast<int>(need);
+    // variants (tools/tune_mandel.py): {lanes per row, vote interval}
+    const int v = launch_override().per_thread;
+    switch (v) {
+        case 2: return launch_t<4, 16>(a, stream);
+        case 3: return launch_t<4, 8>(a, stream);
+        case 4: return launch_t<8, 8>(a, stream);
+        case 5: return launch_t<16, 16>(a, stream);
+        case 6: return launch_t<8, 32>(a, stream);
+        default: return launch_t<8, 16>(a, stream);
     }
-    a.total_warps = static_cast<unsigned>(grid) * 8u;
-    mandel_kernel<<<grid, 256, 0, stream>>>(a);
-    return cudaGetLastError();
 }
 
 }  // namespace mandel
