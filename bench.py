@@ -159,8 +159,15 @@ def dist_init(args):
     if world > 1 and not dist.is_initialized():
         if args.impl == "reference":
             return rank, world, local
+        # LIME_DIST_BACKEND=gloo lets several ranks share one GPU to exercise the multi-rank code
+        # path where only one GPU is available (NCCL needs one GPU per rank); not for timing.
+        backend = os.environ.get("LIME_DIST_BACKEND", "nccl")
+        local = local % max(torch.cuda.device_count(), 1)
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     elif torch.cuda.is_available():
         torch.cuda.set_device(local)
     return rank, world, local
@@ -236,7 +243,7 @@ def run_nbody(args, rank, world, local):
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": "BASELINE.json configs[4]: N-body all-pairs 2^20 bodies fp32, index-space "
+            "config": {"workload": f"BASELINE.json configs[4]: N-body all-pairs {n} bodies fp32, index-space "
                                    "sharded, NCCL all-gather per step",
                        "n_bodies": n, "eps2": EPS2, "dt": DT, "targets_per_gpu": sim.count,
                        "parallelism": f"target-index shards x{world}" + (" + all_gather" if world > 1 else ""),
@@ -474,7 +481,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["lime", "reference"], default="lime")
-    ap.add_argument("--n", type=int, default=1 << 20)
+    ap.add_argument("--bodies", dest="n", type=int, default=1 << 20)
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--cpu-targets", type=int, default=3072)
     ap.add_argument("--ref-targets", type=int, default=512)
