@@ -72,6 +72,18 @@ template <> struct Policy<kMax, int32_t> : MinMaxI<int32_t, INT_MIN, false> {};
 template <> struct Policy<kMin, int64_t> : MinMaxI<int64_t, LLONG_MAX, true> {};
 template <> struct Policy<kMax, int64_t> : MinMaxI<int64_t, LLONG_MIN, false> {};
 
+// L2 (coherent) load of a CTA partial written by another CTA
+template <typename A>
+__device__ __forceinline__ A ldcg_acc(const A* p) {
+    if constexpr (sizeof(A) == 8) {
+        const unsigned long long v = __ldcg(reinterpret_cast<const unsigned long long*>(p));
+        return *reinterpret_cast<const A*>(&v);
+    } else {
+        const unsigned v = __ldcg(reinterpret_cast<const unsigned*>(p));
+        return *reinterpret_cast<const A*>(&v);
+    }
+}
+
 template <typename P, typename A>
 __device__ __forceinline__ A warp_reduce(A v) {
 #pragma unroll
@@ -114,7 +126,18 @@ __global__ void __launch_bounds__(256) reduce_kernel(const T* __restrict__ x, in
     int64_t i = gtid;
     for (; i + 3 * stride < nv; i += 4 * stride) {   // 4 independent 128-bit loads in flight
         const uint4 r0 = ldv(i), r1 = ldv(i + stride), r2 = ldv(i + 2 * stride), r3 = ldv(i + 3 * stride);
-        fold(r0); fold(r1); fold(r2); fold(r3);
+        if constexpr (OP == kSum && std::is_same<T, float>::value) {
+            // fp32 sums: add the 16 loaded elements in fp32 and widen once -- F2F.F64.F32 runs at
+            // ~8 lanes/clk/SM (profiles/microbench), so one conversion per element would cap the
+            // kernel below HBM speed.
+            const float4 a = reinterpret_cast<const float4&>(r0), b = reinterpret_cast<const float4&>(r1);
+            const float4 c = reinterpret_cast<const float4&>(r2), d = reinterpret_cast<const float4&>(r3);
+            const float s16 = (((a.x + a.y) + (a.z + a.w)) + ((b.x + b.y) + (b.z + b.w))) +
+                              (((c.x + c.y) + (c.z + c.w)) + ((d.x + d.y) + (d.z + d.w)));
+            acc = P::comb(acc, P::lift(s16));
+        } else {
+            fold(r0); fold(r1); fold(r2); fold(r3);
+        }
     }
     for (; i < nv; i += stride) fold(ldv(i));
     if (gtid < n - tail0) acc = P::comb(acc, P::lift(x[tail0 + gtid]));
@@ -133,16 +156,19 @@ __global__ void __launch_bounds__(256) reduce_kernel(const T* __restrict__ x, in
     __syncthreads();
     if (!s_last) return;
     __threadfence();
-    if (threadIdx.x == 0) {
-        // fixed CTA-index order (deterministic)
-        volatile A* vp = partial;
-        A b = vp[0];
-        for (unsigned k = 1; k < gridDim.x; ++k) b = P::comb(b, vp[k]);
-        if constexpr (OP != kSum && std::is_floating_point<T>::value) {
-            if (n == 0) b = (OP == kMin) ? static_cast<A>(INFINITY) : static_cast<A>(-INFINITY);  // R9
+    if (warp == 0) {
+        // fixed order (deterministic for a given grid): lane l folds partials l, l+32, ... in index
+        // order, then the fixed xor-shuffle tree combines the 32 lane values
+        A b = P::id();
+        for (unsigned k = lane_id(); k < gridDim.x; k += 32) b = P::comb(b, ldcg_acc(partial + k));
+        b = warp_reduce<P>(b);
+        if (lane_id() == 0) {
+            if constexpr (OP != kSum && std::is_floating_point<T>::value) {
+                if (n == 0) b = (OP == kMin) ? static_cast<A>(INFINITY) : static_cast<A>(-INFINITY);  // R9
+            }
+            *out = static_cast<T>(b);
+            *ticket = 0u;
         }
-        *out = static_cast<T>(b);
-        *ticket = 0u;
     }
 }
 

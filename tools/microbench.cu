@@ -128,6 +128,27 @@ __global__ void k_rcp(float* out, float a, float b, int iters) {
     if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
 }
 
+// FFMA2 whose three operands are distinct register pairs (the N-Body accumulate shape) vs the
+// uniform-operand FFMA2 above: exposes register-file bank limits of 6-register FFMA2 reads.
+__global__ void k_ffma2_3reg(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float2 x[CH], p[CH], q[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) {
+        x[c] = make_float2(threadIdx.x * 1e-3f + c, c);
+        p[c] = make_float2(a + c * 1e-3f, a - c * 1e-3f);
+        q[c] = make_float2(b * c, b + c);
+    }
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = ffma2(p[c], q[c], x[c]);
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c].x + x[c].y;
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+
 __global__ void k_dfma(float* out, float a, float b, int iters) {
     long long t0 = clock64();
     double x[CH];
@@ -237,6 +258,7 @@ int main() {
     struct { const char* name; void (*k)(float*, float, float, int); double lane_ops_per_iter; } tests[] = {
         {"ffma", k_ffma, CH}, {"ffma2", k_ffma2, 2.0 * CH}, {"fadd2", k_fadd2, 2.0 * CH},
         {"mufu_rsq", k_rsq, CH}, {"mufu_ex2(+fmul)", k_ex2, CH},
+        {"ffma2_3reg_pairs", k_ffma2_3reg, 2.0 * CH},
         {"mufu_lg2(+fadd)", k_lg2, CH}, {"mufu_rcp", k_rcp, CH},
         {"dfma(fp64 lanes)", k_dfma, CH}, {"ffma2+dfma(fp32 lanes only)", k_mix, 2.0 * CH},
         {"f32->f64->f32 roundtrips(+dmul)", k_f2d, CH},
