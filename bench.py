@@ -300,6 +300,18 @@ def run_extras(peaks, flush):
                          "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s", "frac": ach / fp32,
                                       "traffic": ncu_traffic("nbody_force_4096")}}
     del b, acc
+    # the same step in a simulation loop: 100 force + integrate steps captured in one CUDA graph
+    sim4k = ldist.NBodySim(torch.from_numpy(inputs.nbody_bodies(4096, seed=1)), EPS2, DT, "cuda")
+    g4k = sim4k.capture(100)
+    med, _ = time_launches(g4k.replay, 10, 2, flush)
+    out["nbody_4096_graph"] = {"workload": "configs[0]: N-body 4096, 100 steps (force + integrator) per CUDA-graph replay",
+                               "value": inter * 100 / (med * 1e-3), "unit": "interactions/s",
+                               "ms_per_step": med / 100,
+                               "roofline": {"bound": "alu", "achieved": FLOP_PER_INTERACTION * inter * 100 / (med * 1e-3) / 1e12,
+                                            "peak": fp32, "unit": "TFLOP/s",
+                                            "frac": FLOP_PER_INTERACTION * inter * 100 / (med * 1e-3) / 1e12 / fp32,
+                                            "traffic": None}}
+    del sim4k, g4k
 
     # config 2: Black-Scholes 2^24 options: map (20 B/option) and fused map+reduce (12 B/option)
     n = 1 << 24

@@ -291,12 +291,13 @@ __device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
 struct Params2 {
     float* C;
     int M, N, K;
+    int group;                 // raster group: pair-tile rows that sweep the N tiles together
     int num_m, num_n, num_k;   // num_m counts 256-row pair tiles
     int num_tiles;
 };
 
 __device__ __forceinline__ void tile_coords2(int t, const Params2& p, int& mb, int& nb) {
-    constexpr int G = 8;       // raster group of pair-tile rows sharing Bt tiles in L2
+    const int G = p.group;     // raster group of pair-tile rows sharing Bt tiles in L2
     const int per_group = G * p.num_n;
     const int g = t / per_group;
     const int first_m = g * G;
@@ -483,6 +484,7 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
         p.num_n = static_cast<int>(ceil_div<int64_t>(N, two::BN));
         p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
         p.num_tiles = p.num_m * p.num_n;
+        p.group = ov.block_threads > 0 ? ov.block_threads : 8;   // override: raster group (sweep)
         static bool attr2 = false;
         if (!attr2) {
             cudaError_t e = cudaFuncSetAttribute(gemm2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,

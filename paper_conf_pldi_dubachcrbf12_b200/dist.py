@@ -85,6 +85,23 @@ class NBodySim:
         h_pos.copy_(self.pos, non_blocking=True)
         h_vel.copy_(self.vel, non_blocking=True)
 
+    def capture(self, steps: int) -> "torch.cuda.CUDAGraph":
+        """Capture `steps` simulation steps into one CUDA graph (single rank only). The kernels take
+        no host decisions and their workspaces self-reset, so a replay runs the steps back to back
+        without launch gaps -- the paper's repeated task-graph passes (L113-114) as one launch."""
+        if self.world != 1:
+            raise RuntimeError("graph capture of the multi-rank step (NCCL inside the graph) is not supported")
+        s = torch.cuda.Stream(self.device)
+        s.wait_stream(torch.cuda.current_stream(self.device))
+        with torch.cuda.stream(s):
+            self.step()                      # warm-up on the capture stream (workspace, lazy init)
+        torch.cuda.current_stream(self.device).wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(steps):
+                self.step()
+        return g
+
     def momentum(self) -> torch.Tensor:
         """Global sum of m v over all ranks (all_reduce), float64 [3]."""
         m = self.pos[:, 3:4].double()

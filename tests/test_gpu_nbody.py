@@ -162,3 +162,17 @@ def test_nbody_f64_shards_and_config5_sample(lime):
     ref = np.stack([oracle.nbody_accel_f64(b, 1e-4, int(r), 1, with_mag=True)[0][0] for r in rows])
     mag = np.array([oracle.nbody_accel_f64(b, 1e-4, int(r), 1, with_mag=True)[1][0] for r in rows])
     assert nbody_rel_err(full.numpy()[rows], ref, mag).max() <= NBODY64_RTOL
+
+
+def test_cuda_graph_replay_matches_eager_steps(lime):
+    from paper_conf_pldi_dubachcrbf12_b200 import dist as ldist
+    n, steps = 4096, 5
+    bodies = torch.from_numpy(inputs.nbody_bodies(n, seed=61))
+    eager = ldist.NBodySim(bodies, 1e-4, 1e-3, "cuda:0")
+    for _ in range(steps + 1):                      # capture() runs one warm-up step first
+        eager.step()
+    sim = ldist.NBodySim(bodies, 1e-4, 1e-3, "cuda:0")
+    g = sim.capture(steps)
+    g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(sim.pos, eager.pos) and torch.equal(sim.vel, eager.vel)
