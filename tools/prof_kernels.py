@@ -3,7 +3,8 @@
     ncu --set full --clock-control none --import-source on -k regex:<kernel> -s 1 -c 1 \
         -o gpurun_out/prof_<which> python tools/prof_kernels.py <which>
 
-which: nbody1m | nbody1m_p8 | nbody4096 | bs_map | bs_fused | mandel | matmul | reduce | cp | mriq
+which: nbody1m | nbody1m_p8 | nbody4096 | nbody64 | bs_map | bs_fused | mandel | matmul | reduce | cp | mriq
+       | series | idea
 """
 import os
 import sys
@@ -52,6 +53,18 @@ def main(which: str, reps: int = 3):
         vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
         for _ in range(reps):
             lime.map_mriq(k, vx)
+    elif which == "nbody64":
+        b = torch.from_numpy(inputs.nbody_bodies(1 << 20, seed=5).astype(np.float64)).cuda()
+        for _ in range(reps):
+            lime.map_nbody_f64(b, 1e-4, 0, 1 << 17)     # bench.py's nbody_f64 shape
+    elif which == "series":
+        for _ in range(reps):
+            lime.map_series(0, inputs.SERIES_N)
+    elif which == "idea":
+        data = torch.from_numpy(inputs.crypt_data()).cuda()
+        ek, _ = lime.idea_key_schedule(inputs.crypt_key())
+        for _ in range(reps):
+            lime.map_idea(data, ek)
     elif which == "reduce":
         x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
         for _ in range(reps):
