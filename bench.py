@@ -312,6 +312,17 @@ def run_extras(peaks, flush):
                                             "frac": FLOP_PER_INTERACTION * inter * 100 / (med * 1e-3) / 1e12 / fp32,
                                             "traffic": None}}
     del sim4k, g4k
+    # ... and as one persistent cooperative launch (lime_nbody_simulate: grid barrier between steps)
+    p4k = torch.from_numpy(inputs.nbody_bodies(4096, seed=1)).cuda()
+    v4k = torch.zeros_like(p4k)
+    med, _ = time_launches(lambda: lime.nbody_simulate(p4k, v4k, 100, EPS2, DT), 10, 2, flush)
+    ach = FLOP_PER_INTERACTION * inter * 100 / (med * 1e-3) / 1e12
+    out["nbody_4096_simulate"] = {"workload": "configs[0]: N-body 4096, 100 steps (force + integrator) in one persistent launch",
+                                  "value": inter * 100 / (med * 1e-3), "unit": "interactions/s",
+                                  "ms_per_step": med / 100,
+                                  "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s",
+                                               "frac": ach / fp32, "traffic": None}}
+    del p4k, v4k
 
     # config 2: Black-Scholes 2^24 options: map (20 B/option) and fused map+reduce (12 B/option)
     n = 1 << 24

@@ -137,11 +137,25 @@ lime_status lime_map_nbody_f64(const double *bodies, int64_t n_src, int64_t tgt_
 lime_status lime_map_nbody_integrate(float *pos, float *vel, const float *accel, int64_t n,
                                      float dt, void *stream);
 
+/* `steps` complete N-Body simulation steps on DEVICE buffers (the paper's task
+ * graph run repeatedly, `particles => computeForces => forceAccumulator`,
+ * PAPER.md L106-114; its 4096-body size, Table 3): per step the force map
+ * over all n targets against all n sources, then the integrator, with results
+ * bit-identical to `steps` x (lime_map_nbody(pos, n, 0, n, ...) +
+ * lime_map_nbody_integrate). pos, vel: [n][4] float, device, 16-B aligned,
+ * disjoint, updated in place. n <= 8192: one persistent cooperative launch (all
+ * CTAs resident, a grid barrier between steps, positions ping-ponged through
+ * ws); larger n: one force + one integrator launch per step. Do not run two
+ * calls sharing one ws concurrently (the grid barrier lives in ws).
+ * ws: lime_nbody_simulate_workspace_bytes(n) bytes, device, zero-filled once. */
+size_t lime_nbody_simulate_workspace_bytes(int64_t n);
+lime_status lime_nbody_simulate(float *pos, float *vel, int64_t n, int32_t steps, float eps2,
+                                float dt, void *ws, size_t ws_bytes, void *stream);
+
 /* One complete N-Body simulation step through HOST buffers (end-to-end entry,
  * PAPER.md Fig. 6 / §4.3 L275-286 host<->device transport): copies h_pos and
  * h_vel ([n][4] float, host memory, pinned for best speed) to the device
- * scratch `ws`, runs `steps` x (lime_map_nbody over all n targets +
- * lime_map_nbody_integrate), copies the new state back into h_pos / h_vel and
+ * scratch `ws`, runs lime_nbody_simulate(steps) on them, copies the new state back into h_pos / h_vel and
  * synchronises `stream`. ws: lime_nbody_simulate_host_workspace_bytes(n) bytes,
  * device, zero-filled before first use. */
 size_t lime_nbody_simulate_host_workspace_bytes(int64_t n);

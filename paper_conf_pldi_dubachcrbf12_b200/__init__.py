@@ -7,7 +7,7 @@ workspaces. Every step of the path runs in the CUDA kernels; there is no CPU fal
 library is missing, load() raises.
 
 Public API (names follow the ABI):
-    map_nbody, map_nbody_integrate, nbody_simulate_host,
+    map_nbody, map_nbody_integrate, nbody_simulate, nbody_simulate_host,
     map_blackscholes, map_reduce_blackscholes_sum,
     map_mandelbrot, map_matmul_bf16,
     reduce_sum / reduce_min / reduce_max (f32, f64, i32, i64),
@@ -54,6 +54,8 @@ SIGNATURES = {
     "lime_map_nbody_integrate": (_int, [_p, _p, _p, _i64, _f, _p]),
     "lime_map_nbody_f64_workspace_bytes": (_sz, [_i64, _i64]),
     "lime_map_nbody_f64": (_int, [_p, _i64, _i64, _i64, C.c_double, _p, _p, _sz, _p]),
+    "lime_nbody_simulate_workspace_bytes": (_sz, [_i64]),
+    "lime_nbody_simulate": (_int, [_p, _p, _i64, _i32, _f, _f, _p, _sz, _p]),
     "lime_nbody_simulate_host_workspace_bytes": (_sz, [_i64]),
     "lime_nbody_simulate_host": (_int, [_p, _p, _i64, _i32, _f, _f, _p, _sz, _p]),
     "lime_map_blackscholes": (_int, [_p, _p, _p, _i64, _f, _f, _p, _p, _p]),
@@ -206,6 +208,20 @@ def map_nbody_integrate(pos: torch.Tensor, vel: torch.Tensor, accel: torch.Tenso
         _dev_tensor(t, torch.float32, nm, 4)
     _check(L.lime_map_nbody_integrate(pos.data_ptr(), vel.data_ptr(), accel.data_ptr(), pos.shape[0], dt,
                                       _stream(pos.device)), "lime_map_nbody_integrate")
+
+
+def nbody_simulate(pos: torch.Tensor, vel: torch.Tensor, steps: int, eps2: float, dt: float) -> None:
+    """`steps` force+integrate steps on device state pos/vel ([n][4] float32, updated in place); one
+    persistent launch for n <= 8192."""
+    L = load()
+    _dev_tensor(pos, torch.float32, "pos", 4)
+    _dev_tensor(vel, torch.float32, "vel", 4)
+    if vel.shape[0] != pos.shape[0] or vel.device != pos.device:
+        raise ValueError("pos and vel must have the same length and device")
+    n = pos.shape[0]
+    ws = workspace(pos.device, "nbody_sim", L.lime_nbody_simulate_workspace_bytes(n))
+    _check(L.lime_nbody_simulate(pos.data_ptr(), vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(), ws.numel(),
+                                 _stream(pos.device)), "lime_nbody_simulate")
 
 
 def nbody_simulate_host(h_pos: torch.Tensor, h_vel: torch.Tensor, steps: int, eps2: float, dt: float,

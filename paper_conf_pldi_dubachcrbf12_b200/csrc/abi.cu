@@ -207,17 +207,46 @@ lime_status lime_map_nbody_integrate(float* pos, float* vel, const float* accel,
                     "lime_map_nbody_integrate");
 }
 
-// ws layout: [pos n*16][vel n*16][accel n*16][nbody workspace]
+static lime_status sim_validate(const char* fn, int64_t n, int32_t steps, float eps2, float dt) {
+    if (n < 0 || steps < 0) return fail(LIME_ERR_INVALID_ARG, "%s: n or steps < 0", fn);
+    if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f) || !std::isfinite(dt))
+        return fail(LIME_ERR_INVALID_ARG, "%s: bad eps2 or dt", fn);
+    return LIME_OK;
+}
+
+size_t lime_nbody_simulate_workspace_bytes(int64_t n) {
+    if (n < 0) return 0;
+    return nbody::simulate_workspace_bytes(n);
+}
+
+lime_status lime_nbody_simulate(float* pos, float* vel, int64_t n, int32_t steps, float eps2, float dt, void* ws,
+                                size_t ws_bytes, void* stream) {
+    LIME_TRY(sim_validate("lime_nbody_simulate", n, steps, eps2, dt));
+    if (n == 0) return LIME_OK;
+    if (!pos || !vel || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate: null pointer");
+    if (!aligned16(pos) || !aligned16(vel) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_nbody_simulate: pos, vel, ws must be 16-byte aligned");
+    const size_t b = static_cast<size_t>(n) * 16;
+    if (overlap(pos, b, vel, b) || overlap(ws, ws_bytes, pos, b) || overlap(ws, ws_bytes, vel, b))
+        return fail(LIME_ERR_ALIASING, "lime_nbody_simulate: pos, vel and ws must be disjoint");
+    LIME_TRY(check_device());
+    if (ws_bytes < lime_nbody_simulate_workspace_bytes(n))
+        return fail(LIME_ERR_WORKSPACE, "lime_nbody_simulate: workspace too small");
+    return launched(nbody::launch_simulate(reinterpret_cast<float4*>(pos), reinterpret_cast<float4*>(vel), n, steps,
+                                           eps2, dt, ws, static_cast<cudaStream_t>(stream)),
+                    "lime_nbody_simulate");
+}
+
+// ws layout: [simulate workspace (zero-invariant words at fixed offsets)][pos n*16][vel n*16]
+static size_t sim_host_state_offset(int64_t n) { return ((nbody::simulate_workspace_bytes(n) + 255) / 256) * 256; }
 size_t lime_nbody_simulate_host_workspace_bytes(int64_t n) {
     if (n < 0) return 0;
-    return static_cast<size_t>(n) * 48 + nbody::workspace_bytes(n, n);
+    return sim_host_state_offset(n) + static_cast<size_t>(n) * 32;
 }
 
 lime_status lime_nbody_simulate_host(float* h_pos, float* h_vel, int64_t n, int32_t steps, float eps2, float dt,
                                      void* ws, size_t ws_bytes, void* stream) {
-    if (n < 0 || steps < 0) return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: n or steps < 0");
-    if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f) || !std::isfinite(dt))
-        return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: bad eps2 or dt");
+    LIME_TRY(sim_validate("lime_nbody_simulate_host", n, steps, eps2, dt));
     if (n == 0) return LIME_OK;
     if (!h_pos || !h_vel || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_nbody_simulate_host: null pointer");
     if (!aligned16(ws)) return fail(LIME_ERR_MISALIGNED, "lime_nbody_simulate_host: ws must be 16-byte aligned");
@@ -228,16 +257,12 @@ lime_status lime_nbody_simulate_host(float* h_pos, float* h_vel, int64_t n, int3
         return fail(LIME_ERR_WORKSPACE, "lime_nbody_simulate_host: workspace too small");
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     char* w = static_cast<char*>(ws);
-    float4* d_pos = reinterpret_cast<float4*>(w);
-    float4* d_vel = reinterpret_cast<float4*>(w + b);
-    float4* d_acc = reinterpret_cast<float4*>(w + 2 * b);
-    void* d_ws = w + 3 * b;
+    void* d_ws = w;
+    float4* d_pos = reinterpret_cast<float4*>(w + sim_host_state_offset(n));
+    float4* d_vel = reinterpret_cast<float4*>(w + sim_host_state_offset(n) + b);
     cudaError_t e = cudaMemcpyAsync(d_pos, h_pos, b, cudaMemcpyHostToDevice, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(d_vel, h_vel, b, cudaMemcpyHostToDevice, s);
-    for (int32_t k = 0; k < steps && e == cudaSuccess; ++k) {
-        e = nbody::launch_force(d_pos, n, 0, n, eps2, d_acc, d_ws, s);
-        if (e == cudaSuccess) e = nbody::launch_integrate(d_pos, d_vel, d_acc, n, dt, s);
-    }
+    if (e == cudaSuccess) e = nbody::launch_simulate(d_pos, d_vel, n, steps, eps2, dt, d_ws, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(h_pos, d_pos, b, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(h_vel, d_vel, b, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);

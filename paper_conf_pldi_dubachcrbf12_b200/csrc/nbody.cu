@@ -284,6 +284,23 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
 // =====================================================================================
 constexpr int64_t kSmallMaxSources = 8192;
 
+// One split's contribution for one target: chunk partials added into the split accumulator in chunk
+// order -- the arithmetic of force_kernel's scalar variant (shared by force_small_kernel and the
+// persistent simulation kernel, so all three agree bit for bit).
+__device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* sb, int len, float eps2) {
+    for (int c0 = 0; c0 < len; c0 += kChunk) {
+        const int c1 = mn(len, c0 + kChunk);
+        it.chunk_begin();
+        if (c1 - c0 == kChunk) {
+#pragma unroll 4
+            for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
+        } else {
+            for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+        }
+        it.chunk_end();
+    }
+}
+
 __global__ void __launch_bounds__(32 * kMaxSplits) force_small_kernel(const __grid_constant__ ForceArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                          // [S][split_len]
@@ -310,18 +327,7 @@ __global__ void __launch_bounds__(32 * kMaxSplits) force_small_kernel(const __gr
     }
     __syncwarp();
     mbar_wait(&bar[warp], 0);
-    const float eps2 = a.eps2;
-    for (int c0 = 0; c0 < len; c0 += kChunk) {
-        const int c1 = mn(len, c0 + kChunk);
-        it.chunk_begin();
-        if (c1 - c0 == kChunk) {
-#pragma unroll 4
-            for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
-        } else {
-            for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
-        }
-        it.chunk_end();
-    }
+    split_sum(it, sb, len, a.eps2);
     part[warp * 32 + lane] = it.result(0);
     __syncthreads();
     if (warp == 0 && valid) {
@@ -349,6 +355,175 @@ static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
     return cudaGetLastError();
 }
 
+// =====================================================================================
+// Whole simulation in one persistent launch (n <= kSmallMaxSources; the paper's repeated
+// task-graph pass, at its own 4096-body size, Table 3). At this size a
+// step is a few microseconds of FP32 work, so launch gaps and a separate integrator pass cost as
+// much as the forces. One cooperative grid (every CTA resident) runs all `steps`: per step each
+// warp stages its source split from the current position buffer (L2, ld.global.cg), each CTA
+// computes the forces on its 32-target groups exactly as force_small_kernel does, and warp 0
+// applies the integrator (integrate_kernel's arithmetic) and writes the new positions into the
+// other buffer; then a grid barrier. Positions ping-pong between `pos` and a workspace copy; a
+// velocity is only ever touched by its target's thread. Bit-identical to `steps` x
+// (lime_map_nbody + lime_map_nbody_integrate).
+// (A CTA-pair variant -- clusters of 2, one packed target pair per lane, split partials combined
+// through DSMEM -- was measured slower at 4096: 1024 packed warps leave ~2 per SM sub-partition,
+// too few to hide the dependent FFMA2/MUFU chains; see profiles/experiments.)
+// =====================================================================================
+struct SimArgs {
+    float4* pos;        // [n] in/out
+    float4* vel;        // [n] in/out
+    float4* pos_alt;    // [n] workspace
+    unsigned* bar;      // [2] grid barrier arrivals, exits (zero between launches)
+    int64_t n;
+    int32_t steps;
+    int32_t splits;
+    int64_t split_len;
+    float eps2, dt;
+};
+
+__device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(arrivals) : "memory");
+        unsigned v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(arrivals) : "memory");
+        } while (v < target);
+    }
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(32 * kMaxSplits) simulate_small_kernel(const __grid_constant__ SimArgs a) {
+    extern __shared__ __align__(128) uint8_t small_smem[];
+    float4* src = reinterpret_cast<float4*>(small_smem);                                   // [S][split_len]
+    float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
+    const int warp = threadIdx.x >> 5;                // = split index
+    const unsigned lane = lane_id();
+    const int64_t groups = ceil_div<int64_t>(a.n, 32);
+    const int64_t j0 = static_cast<int64_t>(warp) * a.split_len;
+    const int len = static_cast<int>(mn<int64_t>(a.n, j0 + a.split_len) - j0);
+    float4* sb = src + j0;
+    unsigned barrier_target = 0;
+
+    for (int32_t k = 0; k < a.steps; ++k) {
+        const float4* cur = (k & 1) ? a.pos_alt : a.pos;
+        float4* nxt = (k & 1) ? a.pos : a.pos_alt;
+        for (int j = static_cast<int>(lane); j < len; j += 32) sb[j] = __ldcg(cur + j0 + j);
+        __syncwarp();
+        for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
+            const int64_t t = g * 32 + lane;
+            const bool valid = t < a.n;
+            const float4 p = __ldcg(cur + (valid ? t : a.n - 1));
+            Interact<1, false> it;
+            it.set(0, p);
+            it.zero_all();
+            split_sum(it, sb, len, a.eps2);
+            part[warp * 32 + lane] = it.result(0);
+            __syncthreads();
+            if (warp == 0 && valid) {
+                float4 acc = part[lane];
+                for (int s = 1; s < a.splits; ++s) {
+                    const float4 q = part[s * 32 + lane];
+                    acc.x += q.x; acc.y += q.y; acc.z += q.z;
+                }
+                float4 v = a.vel[t];
+                float4 pn = p;
+                v.x = fmaf(acc.x, a.dt, v.x);
+                v.y = fmaf(acc.y, a.dt, v.y);
+                v.z = fmaf(acc.z, a.dt, v.z);
+                pn.x = fmaf(v.x, a.dt, pn.x);
+                pn.y = fmaf(v.y, a.dt, pn.y);
+                pn.z = fmaf(v.z, a.dt, pn.z);
+                a.vel[t] = v;
+                __stcg(nxt + t, pn);
+            }
+            __syncthreads();                       // part[] is reused by the next group
+        }
+        const bool last = (k + 1 == a.steps);
+        if (!last || (a.steps & 1)) {
+            barrier_target += gridDim.x;
+            grid_barrier(a.bar, barrier_target);
+        }
+    }
+    if ((a.steps & 1) && warp == 0) {              // final positions are in pos_alt: copy own targets back
+        for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
+            const int64_t t = g * 32 + lane;
+            if (t < a.n) a.pos[t] = __ldcg(a.pos_alt + t);
+        }
+    }
+    if (threadIdx.x == 0) {                        // the last CTA out leaves the barrier zeroed
+        __threadfence();
+        if (atomicAdd(a.bar + 1, 1u) == gridDim.x - 1) {
+            a.bar[0] = 0u;
+            a.bar[1] = 0u;
+        }
+    }
+}
+
+// workspace: [grid barrier, 256 B][force workspace (its tickets first)][pos_alt / accel, n x 16 B] --
+// every zero-invariant word sits at an offset that does not depend on n, so a workspace reused
+// across sizes stays valid.
+static size_t simulate_alt_offset(int64_t n) { return 256 + ((workspace_bytes(n, n) + 255) / 256) * 256; }
+size_t simulate_workspace_bytes(int64_t n) { return simulate_alt_offset(n) + static_cast<size_t>(n) * 16; }
+
+cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, float eps2, float dt, void* ws,
+                            cudaStream_t stream) {
+    if (n == 0 || steps == 0) return cudaSuccess;
+    char* w = static_cast<char*>(ws);
+    float4* alt = reinterpret_cast<float4*>(w + simulate_alt_offset(n));   // pos_alt (persistent) / accel (loop)
+    void* fws = w + 256;
+    if (n > kSmallMaxSources) {                                  // one force + integrate launch per step
+        for (int32_t k = 0; k < steps; ++k) {
+            cudaError_t e = launch_force(pos, n, 0, n, eps2, alt, fws, stream);
+            if (e == cudaSuccess) e = launch_integrate(pos, vel, alt, n, dt, stream);
+            if (e != cudaSuccess) return e;
+        }
+        return cudaSuccess;
+    }
+    SimArgs a;
+    a.pos = pos;
+    a.vel = vel;
+    a.pos_alt = alt;
+    a.bar = reinterpret_cast<unsigned*>(w);
+    a.n = n;
+    a.steps = steps;
+    a.splits = splits(n);
+    a.split_len = chunks_per_split(n) * kChunk;
+    a.eps2 = eps2;
+    a.dt = dt;
+    const int block = 32 * a.splits;
+    const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(simulate_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplits * 32 * 16));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    int occ = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, simulate_small_kernel, block, smem);
+    if (e != cudaSuccess) return e;
+    if (occ < 1) return cudaErrorInvalidConfiguration;
+    const int64_t groups = ceil_div<int64_t>(n, 32);
+    int grid = static_cast<int>(mn<int64_t>(groups, static_cast<int64_t>(occ) * device_num_sms()));
+    const LaunchOverride& ov = launch_override();
+    if (ov.grid_ctas > 0) grid = static_cast<int>(mn<int64_t>(grid, ov.grid_ctas));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(static_cast<unsigned>(grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(block));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeCooperative;         // all CTAs co-resident (the grid barrier needs it)
+    at[0].val.cooperative = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, simulate_small_kernel, a);
+    if (e != cudaSuccess) return e;
+    return cudaGetLastError();
+}
 // =====================================================================================
 // Staging ablation (the paper's Fig. 8: the same kernel with the
 // broadcast array mapped to global, local, texture or constant memory, with or without

@@ -273,9 +273,14 @@ size_t cp_workspace_bytes(int64_t n_atoms, int64_t points) {
     return counters_bytes(points) + (splits(n_atoms) > 1 ? static_cast<size_t>(splits(n_atoms)) * points * 4 : 0) + 256;
 }
 
+// MRI-Q workspace: [counters][split partials][phiMag table]. The counters sit at offset 0 whatever the
+// sizes, so a workspace reused with other sizes still has zeroed counters where the next call looks.
+static size_t mriq_table_offset(int64_t n_k, int64_t n_x) {
+    const size_t b = counters_bytes(n_x) + (splits(n_k) > 1 ? static_cast<size_t>(splits(n_k)) * n_x * 8 : 0);
+    return ((b + 255) / 256) * 256;
+}
 size_t mriq_workspace_bytes(int64_t n_k, int64_t n_x) {
-    const size_t kbytes = ((static_cast<size_t>(n_k) * 16 + 255) / 256) * 256;
-    return kbytes + counters_bytes(n_x) + (splits(n_k) > 1 ? static_cast<size_t>(splits(n_k)) * n_x * 8 : 0) + 256;
+    return mriq_table_offset(n_k, n_x) + static_cast<size_t>(n_k) * 16 + 256;
 }
 
 cudaError_t launch_cp(const float4* atoms, int64_t n_atoms, int32_t nx, int64_t p_begin, int64_t p_count, float z,
@@ -296,8 +301,7 @@ cudaError_t launch_cp(const float4* atoms, int64_t n_atoms, int32_t nx, int64_t 
 cudaError_t launch_mriq(const float* kspace, int64_t n_k, const float* voxels, int64_t x_begin, int64_t x_count,
                         float* out, void* ws, cudaStream_t stream) {
     if (x_count == 0) return cudaSuccess;
-    float4* k4 = static_cast<float4*>(ws);
-    const size_t kbytes = ((static_cast<size_t>(n_k) * 16 + 255) / 256) * 256;
+    float4* k4 = reinterpret_cast<float4*>(static_cast<char*>(ws) + mriq_table_offset(n_k, x_count));
     const int g = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(n_k, 256), 4LL * device_num_sms()));
     phimag_kernel<<<mx(g, 1), 256, 0, stream>>>(kspace, n_k, k4);
     cudaError_t e = cudaGetLastError();
@@ -309,7 +313,7 @@ cudaError_t launch_mriq(const float* kspace, int64_t n_k, const float* voxels, i
     a.tgt_count = x_count;
     a.p.voxels = voxels;
     a.out = reinterpret_cast<float2*>(out);
-    return launch_bmap(a, static_cast<char*>(ws) + kbytes, stream);
+    return launch_bmap(a, ws, stream);
 }
 
 }  // namespace parboil

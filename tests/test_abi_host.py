@@ -30,7 +30,8 @@ def test_header_declares_expected_surface():
     names = declared_functions()
     for must in ("lime_map_nbody", "lime_map_nbody_integrate", "lime_map_blackscholes",
                  "lime_map_reduce_blackscholes_sum", "lime_map_mandelbrot", "lime_map_matmul_bf16",
-                 "lime_reduce_sum_f32", "lime_reduce_max_i64", "lime_nbody_simulate_host"):
+                 "lime_reduce_sum_f32", "lime_reduce_max_i64", "lime_nbody_simulate_host",
+                 "lime_nbody_simulate"):
         assert must in names
 
 
@@ -79,6 +80,23 @@ def test_integrate_and_bs_validation(L):
     assert g(A0, A0 + 4096, A0 + 8192, 16, 0.02, 0.3, A1, A1 + 4096 + 8, None) == 2
     assert g(A0, A0 + 4096, A0 + 8192, 16, 0.02, 0.3, A0 + 4096, A1, None) == 3   # call == X
     assert g(A0, A0 + 4096, A0 + 8192, 0, 0.02, 0.3, A1, A1, None) == 0          # n = 0
+
+
+def test_simulate_validation(L):
+    f = L.lime_nbody_simulate
+    wsb = L.lime_nbody_simulate_workspace_bytes(64)
+    assert wsb >= 64 * 16 + 256
+    assert f(A0, A1, 64, -1, 1e-4, 1e-3, WS, wsb, None) == 1                    # steps < 0
+    assert f(A0, A1, 64, 2, 0.0, 1e-3, WS, wsb, None) == 1                      # eps2 <= 0
+    assert f(A0, A1, 64, 2, 1e-4, float("nan"), WS, wsb, None) == 1             # dt not finite
+    assert f(A0, A1, 0, 2, 1e-4, 1e-3, None, 0, None) == 0                      # n = 0: no-op
+    assert f(A0, None, 64, 2, 1e-4, 1e-3, WS, wsb, None) == 1                   # null vel
+    assert f(A0 + 8, A1, 64, 2, 1e-4, 1e-3, WS, wsb, None) == 2                 # misaligned
+    assert f(A0, A0 + 512, 64, 2, 1e-4, 1e-3, WS, wsb, None) == 3               # pos/vel overlap
+    assert f(A0, A1, 64, 2, 1e-4, 1e-3, A1 + 16, wsb, None) == 3                # ws overlaps vel
+    h = L.lime_nbody_simulate_host
+    assert L.lime_nbody_simulate_host_workspace_bytes(64) >= wsb + 64 * 32
+    assert h(A0, A0 + 64, 8, 1, 1e-4, 1e-3, WS, 1 << 20, None) == 3             # h_pos/h_vel overlap
 
 
 def test_mandelbrot_matmul_reduce_validation(L):

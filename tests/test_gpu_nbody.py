@@ -176,3 +176,56 @@ def test_cuda_graph_replay_matches_eager_steps(lime):
     g.replay()
     torch.cuda.synchronize()
     assert torch.equal(sim.pos, eager.pos) and torch.equal(sim.vel, eager.vel)
+
+
+def _eager_steps(lime, pos, vel, steps, eps2=1e-4, dt=1e-3):
+    for _ in range(steps):
+        a = lime.map_nbody(pos, eps2)
+        lime.map_nbody_integrate(pos, vel, a, dt)
+
+
+@pytest.mark.parametrize("n", [1, 31, 256, 257, 1000, 4096, 8192, 8193])
+def test_simulate_matches_eager_steps(lime, n):
+    # lime_nbody_simulate (one persistent launch for n <= 8192) == steps x (force map + integrator)
+    b = inputs.nbody_bodies(n, seed=70 + n)
+    v0 = (inputs.nbody_bodies(n, seed=71 + n) * np.float32(0.05)).astype(np.float32)
+    v0[:, 3] = 0
+    pos_e, vel_e = _dev(b), _dev(v0)
+    _eager_steps(lime, pos_e, vel_e, 5)
+    pos, vel = _dev(b), _dev(v0)
+    lime.nbody_simulate(pos, vel, 0, 1e-4, 1e-3)                      # no-op
+    assert torch.equal(pos, _dev(b))
+    lime.nbody_simulate(pos, vel, 3, 1e-4, 1e-3)                      # odd: ends in the ping-pong buffer
+    lime.nbody_simulate(pos, vel, 2, 1e-4, 1e-3)                      # barrier words were reset
+    assert torch.equal(pos, pos_e) and torch.equal(vel, vel_e)
+
+
+def test_simulate_grid_independent_and_oracle(lime):
+    n, steps = 4096, 4
+    b = inputs.nbody_bodies(n, seed=80)
+    ref_p, ref_v = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    lime.nbody_simulate(ref_p, ref_v, steps, 1e-4, 1e-3)
+    for g in (1, 7, 64):                                              # CTAs loop over 32-target groups
+        p, v = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+        with lime.launch_override(grid_ctas=g):
+            lime.nbody_simulate(p, v, steps, 1e-4, 1e-3)
+        assert torch.equal(p, ref_p) and torch.equal(v, ref_v), g
+    # one step against the oracle (force, then the integrator)
+    p, v = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    lime.nbody_simulate(p, v, 1, 1e-4, 1e-3)
+    acc, mag = oracle.nbody_accel(b, float(EPS2), with_mag=True)
+    po, vo = oracle.nbody_integrate(b, np.zeros((n, 4), np.float32), np.concatenate([acc, np.zeros((n, 1))], 1), 1e-3)
+    vg = v.cpu().numpy()
+    assert (np.abs(vg[:, :3] - vo[:, :3]).max(axis=1) <= NBODY_RTOL * mag * 1e-3 + 1e-12).all()
+    np.testing.assert_allclose(p.cpu().numpy(), po, rtol=0, atol=2e-7)
+
+
+def test_simulate_host_small_path(lime):
+    n, steps = 4096, 3
+    b = inputs.nbody_bodies(n, seed=81)
+    h_pos = torch.from_numpy(b.copy()).pin_memory()
+    h_vel = torch.zeros((n, 4), dtype=torch.float32).pin_memory()
+    lime.nbody_simulate_host(h_pos, h_vel, steps, 1e-4, 1e-3)
+    pos, vel = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    _eager_steps(lime, pos, vel, steps)
+    assert torch.equal(h_pos, pos.cpu()) and torch.equal(h_vel, vel.cpu())

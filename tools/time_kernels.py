@@ -62,6 +62,14 @@ def main(which):
         vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
         Q = torch.empty((vx.shape[0], 2), device="cuda")
         out["mriq_us"] = 1e3 * time_launches(lambda: lime.map_mriq(k, vx, out=Q), 30, 3, flush)[0]
+    if "series" in which:
+        for dt, nm in ((torch.float32, "f32"), (torch.float64, "f64")):
+            so = torch.empty((inputs.SERIES_N, 2), dtype=dt, device="cuda")
+            out[f"series_{nm}_us"] = 1e3 * time_launches(lambda: lime.map_series(0, inputs.SERIES_N, dtype=dt, out=so), 20, 3, flush)[0]
+    if "sim" in which:
+        p = torch.from_numpy(inputs.nbody_bodies(4096, seed=1)).cuda()
+        v = torch.zeros_like(p)
+        out["sim4096_us_per_step"] = 10 * time_launches(lambda: lime.nbody_simulate(p, v, 100, 1e-4, 1e-3), 10, 2, flush)[0]
     if "reduce" in which:
         x = torch.ones(1 << 28, dtype=torch.float32, device="cuda")
         r = torch.empty((), dtype=torch.float32, device="cuda")
