@@ -5,17 +5,17 @@
 // cos/sin(n pi x) on the same 1001 trapezoid nodes, so the map over n has a broadcast operand: the
 // node table g_i = w_i f(x_i) (w = 1/2 at the ends, 0 at JGF's skipped node x_{m-1}, 1 elsewhere).
 // The phase n pi x_i = 2 pi (n i mod m)/m is reduced EXACTLY in integers, so the trigonometric
-// factors come from an m-entry table of e^{2 pi i p/m} (built per call in fp64, rounded to the
-// variant's precision) -- no range-reduction error at n = 10^5 and no MUFU.
-// B200 form (radix-32 split of the node index, i = 32u + v, g zero-padded to 1024 nodes):
-//   sum_i g_i e^{i theta n i} = sum_u U_u * W_u,  U_u = e^{i theta n 32u},  W_u = sum_v g_{32u+v} V_v,
-//   V_v = e^{i theta n v}.
-// Each thread gathers its coefficient's 32 V_v into REGISTERS (a fully unrolled inner loop indexes
-// them statically), so the 1024 inner terms are one packed FFMA2 each (re and im together) with g
-// read by LDS.128 broadcasts; only the 32 V and 32 U table reads per coefficient are lane-divergent
-// gathers (bank conflicts there cost ~2 % instead of the 2002 conflicting reads per coefficient of
-// the direct form). Every factor is an exactly rounded table value; the one extra rounding per U_u W_u
-// product is bounded by 2 eps sum_u |W_u| <= 2 eps T[|f|].
+// factors come from an m-entry table of e^{2 pi i p/m} (host fp64 libm, rounded to the variant's
+// precision, written once per device) -- no range-reduction error at n = 10^5 and no MUFU.
+// B200 form (radix-R split of the node index, i = R u + v, g zero-padded to 1024 nodes):
+//   sum_i g_i e^{i theta n i} = sum_u U_u * W_u,  U_u = e^{i theta (R n u mod m)},
+//   W_u = sum_v g_{Ru+v} V_v,  V_v = e^{i theta (n v mod m)}.
+// Each thread gathers its coefficient's R values V_v into REGISTERS (a fully unrolled inner loop
+// indexes them statically), so each inner term is one packed FFMA2 (re and im together) whose g
+// operand comes from the kernel-parameter bank (uniform constant loads); only R + 1024/R table reads
+// per coefficient are lane-divergent smem gathers (the direct form did 2002, with 17.7M bank
+// conflicts per launch). Every factor is an exactly rounded table value; the one extra rounding per
+// U_u W_u product is bounded by 2 eps sum_u |W_u| <= 2 eps T[|f|].
 //
 // JG-Crypt (reading R15): IDEA ECB; each thread enciphers 16-byte units (two blocks) with one
 // 128-bit load/store; multiplication modulo 2^16+1 is the branch-free low/high-half form; the 52
@@ -23,35 +23,73 @@
 #include "common.cuh"
 #include "kernels.h"
 
+#include <cmath>
+#include <mutex>
+
 namespace lime {
 namespace jgf {
 
 // ------------------------------------------------------------------ JG-Series
-constexpr int kSeriesM = 1000;   // JGF: TrapezoidIntegrate(0, 2, 1000, ...)
-
-template <typename T>
-__global__ void __launch_bounds__(256) series_tables_kernel(T* g, T* cs, T* sn) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i <= kSeriesM) {
-        const double x = (2.0 / kSeriesM) * i;
-        const double w = (i == 0 || i == kSeriesM) ? 0.5 : (i == kSeriesM - 1 ? 0.0 : 1.0);
-        g[i] = static_cast<T>(w * pow(x + 1.0, x));
-    } else if (i < 1024) {
-        g[i] = 0;                                    // padding nodes of the radix-32 split
-    }
-    if (i < kSeriesM) {
-        double s, c;
-        sincospi(2.0 * i / kSeriesM, &s, &c);   // angle 2 pi i / m
-        cs[i] = static_cast<T>(c);
-        sn[i] = static_cast<T>(s);
-    }
-}
-
-constexpr int kSeriesRadix = 32;          // i = 32 u + v; 32 x 32 = 1024 >= m + 1 nodes
-constexpr int kSeriesNodes = kSeriesRadix * kSeriesRadix;
+constexpr int kSeriesM = 1000;            // JGF: TrapezoidIntegrate(0, 2, 1000, ...)
+constexpr int kSeriesNodes = 1024;        // m + 1 = 1001 nodes, zero-padded
 constexpr int kSeriesBlock = 128;
 
-// (wr, wi) += g * (vr, vi): one FFMA2 in fp32 (bcast g), two DFMA in fp64
+// Node weights g_i = w_i (x_i + 1)^{x_i} (w = 1/2 at the ends, 0 at the skipped node x_{m-1}), rounded
+// to T, as a kernel parameter: the kernel reads them with compile-time offsets, so they arrive through
+// the uniform datapath (LDCU into uniform registers, the FFMA2 broadcast operand) -- A2's constant
+// broadcast (L263-266) -- and never touch shared memory.
+template <typename T>
+struct SeriesNodes {
+    T g[kSeriesNodes];
+};
+
+// e^{2 pi i p / m}, p < m, rounded to T: a per-device constant table written once (host fp64 libm).
+__device__ float d_series_cos32[kSeriesM], d_series_sin32[kSeriesM];
+__device__ double d_series_cos64[kSeriesM], d_series_sin64[kSeriesM];
+
+template <typename T>
+static const SeriesNodes<T>& series_nodes() {
+    static const SeriesNodes<T> nodes = [] {
+        SeriesNodes<T> s{};
+        for (int i = 0; i < kSeriesNodes; ++i) {
+            const double x = (2.0 / kSeriesM) * i;
+            const double w = (i == 0 || i == kSeriesM) ? 0.5 : (i == kSeriesM - 1 ? 0.0 : 1.0);
+            s.g[i] = i <= kSeriesM ? static_cast<T>(w * std::pow(x + 1.0, x)) : T(0);
+        }
+        return s;
+    }();
+    return nodes;
+}
+
+static cudaError_t series_tables_once() {
+    static std::mutex mu;
+    static bool done[256] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lock(mu);
+    if (dev < 0 || dev >= 256) return cudaErrorInvalidDevice;
+    if (done[dev]) return cudaSuccess;
+    static float c32[kSeriesM], s32[kSeriesM];
+    static double c64[kSeriesM], s64[kSeriesM];
+    const double two_pi = 6.283185307179586476925286766559;
+    for (int p = 0; p < kSeriesM; ++p) {
+        // exact symmetries keep the quadrant points exact (cos(pi/2) = 0, ...)
+        const double a = two_pi * p / kSeriesM;
+        c64[p] = (p == 250 || p == 750) ? 0.0 : std::cos(a);
+        s64[p] = (p == 0 || p == 500) ? 0.0 : std::sin(a);
+        c32[p] = static_cast<float>(c64[p]);
+        s32[p] = static_cast<float>(s64[p]);
+    }
+    if ((e = cudaMemcpyToSymbol(d_series_cos32, c32, sizeof c32)) != cudaSuccess) return e;
+    if ((e = cudaMemcpyToSymbol(d_series_sin32, s32, sizeof s32)) != cudaSuccess) return e;
+    if ((e = cudaMemcpyToSymbol(d_series_cos64, c64, sizeof c64)) != cudaSuccess) return e;
+    if ((e = cudaMemcpyToSymbol(d_series_sin64, s64, sizeof s64)) != cudaSuccess) return e;
+    done[dev] = true;
+    return cudaSuccess;
+}
+
+// (wr, wi) += g * (vr, vi): one FFMA2 in fp32 (g broadcast), two DFMA in fp64
 __device__ __forceinline__ float2 cfma(float g, float2 v, float2 w) { return fma2(bcast2(g), v, w); }
 __device__ __forceinline__ double2 cfma(double g, double2 v, double2 w) {
     return make_double2(fma(g, v.x, w.x), fma(g, v.y, w.y));
@@ -59,63 +97,63 @@ __device__ __forceinline__ double2 cfma(double g, double2 v, double2 w) {
 template <typename T> struct Vec2;
 template <> struct Vec2<float> { using type = float2; };
 template <> struct Vec2<double> { using type = double2; };
+template <typename T> __device__ __forceinline__ const T* series_cos();
+template <typename T> __device__ __forceinline__ const T* series_sin();
+template <> __device__ __forceinline__ const float* series_cos<float>() { return d_series_cos32; }
+template <> __device__ __forceinline__ const float* series_sin<float>() { return d_series_sin32; }
+template <> __device__ __forceinline__ const double* series_cos<double>() { return d_series_cos64; }
+template <> __device__ __forceinline__ const double* series_sin<double>() { return d_series_sin64; }
 
-template <typename T>
-__global__ void __launch_bounds__(kSeriesBlock) series_kernel(const T* __restrict__ g, const T* __restrict__ cs,
-                                                              const T* __restrict__ sn, int64_t n0, int64_t count,
-                                                              T* __restrict__ out) {
+// Radix-R split of the node index, i = R u + v: sum_i g_i e^{i theta n i} = sum_u U_u W_u with
+// W_u = sum_v g_{Ru+v} V_v, V_v = e^{i theta (n v mod m)}, U_u = e^{i theta (R n u mod m)}. The V_v live
+// in registers (fully unrolled loops index them statically), g comes from the parameter bank, so each
+// inner term is ONE packed FFMA2 (re and im) and the only lane-divergent accesses are the R + 1024/R
+// table gathers per coefficient. R = 16 for both precisions (measured on B200: fp32 R = 16 at 62 regs,
+// 8 CTAs/SM: 24.7 us vs R = 32 at 96 regs: 28.9 us; fp64 R = 16 at 108 regs: 46.6 us).
+template <typename T, int R>
+__global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_kernel(const __grid_constant__ SeriesNodes<T> G,
+                                                              int64_t n0, int64_t count, T* __restrict__ out) {
     using T2 = typename Vec2<T>::type;
-    __shared__ __align__(16) T sg[kSeriesNodes];
+    constexpr int NU = kSeriesNodes / R;
     __shared__ T sc[kSeriesM], ss[kSeriesM];
-    for (int i = threadIdx.x; i < kSeriesNodes; i += blockDim.x) sg[i] = g[i];      // g[i > m] = 0
-    for (int i = threadIdx.x; i < kSeriesM; i += blockDim.x) { sc[i] = cs[i]; ss[i] = sn[i]; }
+    const T* gc = series_cos<T>();
+    const T* gs = series_sin<T>();
+    for (int i = threadIdx.x; i < kSeriesM; i += blockDim.x) { sc[i] = gc[i]; ss[i] = gs[i]; }
     __syncthreads();
     const T dx = static_cast<T>(2.0 / kSeriesM);
     for (int64_t k = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; k < count;
          k += static_cast<int64_t>(gridDim.x) * blockDim.x) {
         const int64_t n = n0 + k;
         const int step = static_cast<int>(n % kSeriesM);
-        T2 V[kSeriesRadix];                           // V_v = e^{i theta (n v mod m)}
+        T2 V[R];                                      // V_v = e^{i theta (n v mod m)}
         int p = 0;
 #pragma unroll
-        for (int v = 0; v < kSeriesRadix; ++v) {
+        for (int v = 0; v < R; ++v) {
             V[v].x = sc[p];
             V[v].y = ss[p];
             p += step;
             p -= (p >= kSeriesM) ? kSeriesM : 0;
         }
-        const int step_u = p;                         // 32 n mod m
-        int q = 0;                                    // 32 n u mod m
+        const int step_u = p;                         // R n mod m
+        int q = 0;                                    // R n u mod m
         T a = 0, b = 0;
 #pragma unroll 1
-        for (int u = 0; u < kSeriesRadix; ++u) {
+        for (int u = 0; u < NU; ++u) {
+            const T ur = sc[q], ui = ss[q];
+            q += step_u;
+            q -= (q >= kSeriesM) ? kSeriesM : 0;
             T2 w0, w1;                                // W_u, even and odd v (two dependency chains)
             w0.x = w0.y = w1.x = w1.y = 0;
-            const T* gu = sg + u * kSeriesRadix;
 #pragma unroll
-            for (int v = 0; v < kSeriesRadix; v += 4) {
-                T gv[4];
-                if constexpr (sizeof(T) == 4) {
-                    const float4 t = *reinterpret_cast<const float4*>(gu + v);
-                    gv[0] = t.x; gv[1] = t.y; gv[2] = t.z; gv[3] = t.w;
-                } else {
-                    const double2 t0 = *reinterpret_cast<const double2*>(gu + v);
-                    const double2 t1 = *reinterpret_cast<const double2*>(gu + v + 2);
-                    gv[0] = t0.x; gv[1] = t0.y; gv[2] = t1.x; gv[3] = t1.y;
-                }
-                w0 = cfma(gv[0], V[v + 0], w0);
-                w1 = cfma(gv[1], V[v + 1], w1);
-                w0 = cfma(gv[2], V[v + 2], w0);
-                w1 = cfma(gv[3], V[v + 3], w1);
+            for (int v = 0; v < R; ++v) {
+                if (v & 1) w1 = cfma(G.g[u * R + v], V[v], w1);
+                else       w0 = cfma(G.g[u * R + v], V[v], w0);
             }
             const T wr = w0.x + w1.x, wi = w0.y + w1.y;
-            const T ur = sc[q], ui = ss[q];
             a = fma(ur, wr, a);
             a = fma(-ui, wi, a);                      // Re(U W)
             b = fma(ur, wi, b);
             b = fma(ui, wr, b);                       // Im(U W)
-            q += step_u;
-            q -= (q >= kSeriesM) ? kSeriesM : 0;
         }
         if (n == 0) { a = a * static_cast<T>(0.5); b = 0; }   // a_0 = T[f] / 2, b_0 = 0
         out[2 * k + 0] = a * dx;
@@ -123,27 +161,24 @@ __global__ void __launch_bounds__(kSeriesBlock) series_kernel(const T* __restric
     }
 }
 
-size_t series_workspace_bytes(bool f64) { return (f64 ? 8 : 4) * 3 * 1024 + 256; }
+size_t series_workspace_bytes(bool) { return 256; }   // tables are per-device constants now
 
-template <typename T>
-static cudaError_t launch_series_t(int64_t n0, int64_t count, T* out, void* ws, cudaStream_t stream) {
-    T* g = static_cast<T*>(ws);
-    T* cs = g + 1024;
-    T* sn = cs + 1024;
-    series_tables_kernel<T><<<ceil_div(kSeriesNodes, 256), 256, 0, stream>>>(g, cs, sn);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess || count == 0) return e;
+template <typename T, int R>
+static cudaError_t launch_series_t(int64_t n0, int64_t count, T* out, cudaStream_t stream) {
+    if (count == 0) return cudaSuccess;
+    cudaError_t e = series_tables_once();
+    if (e != cudaSuccess) return e;
     int grid = launch_override().grid_ctas;
     if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(count, kSeriesBlock), 16LL * device_num_sms()));
-    series_kernel<T><<<grid, kSeriesBlock, 0, stream>>>(g, cs, sn, n0, count, out);
+    series_kernel<T, R><<<grid, kSeriesBlock, 0, stream>>>(series_nodes<T>(), n0, count, out);
     return cudaGetLastError();
 }
 
-cudaError_t launch_series_f32(int64_t n0, int64_t count, float* out, void* ws, cudaStream_t stream) {
-    return launch_series_t<float>(n0, count, out, ws, stream);
+cudaError_t launch_series_f32(int64_t n0, int64_t count, float* out, void*, cudaStream_t stream) {
+    return launch_series_t<float, 16>(n0, count, out, stream);
 }
-cudaError_t launch_series_f64(int64_t n0, int64_t count, double* out, void* ws, cudaStream_t stream) {
-    return launch_series_t<double>(n0, count, out, ws, stream);
+cudaError_t launch_series_f64(int64_t n0, int64_t count, double* out, void*, cudaStream_t stream) {
+    return launch_series_t<double, 16>(n0, count, out, stream);
 }
 
 // ------------------------------------------------------------------ JG-Crypt (IDEA)
