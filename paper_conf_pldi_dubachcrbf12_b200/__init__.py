@@ -84,7 +84,7 @@ def load(path: str | None = None):
     global _lib
     with _lock:
         if _lib is None:
-            p = path or LIB_PATH
+            p = path or os.environ.get("LIME_LIBRARY") or LIB_PATH   # LIME_LIBRARY: A/B builds (tools/)
             if not os.path.exists(p):
                 raise RuntimeError(f"liblime.so not built ({p}); run `python -m paper_conf_pldi_dubachcrbf12_b200.build`")
             lib = C.CDLL(p)

@@ -97,6 +97,38 @@ __global__ void k_ex2(float* out, float a, float b, int iters) {
     if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
 }
 
+__device__ __forceinline__ float sinf_a(float x) { float y; asm volatile("sin.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
+__device__ __forceinline__ float cosf_a(float x) { float y; asm volatile("cos.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
+// sin.approx = FMUL.RZ (radians -> turns, FMA pipe) + MUFU.SIN; the chain keeps x in [-1, 1]
+__global__ void k_sin(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = 0.3f + threadIdx.x * 1e-6f + c * 1e-3f;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = sinf_a(x[c]);
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+// sin and cos of the same argument (the MRI-Q pattern): 2 MUFU per iteration and channel
+__global__ void k_sincos(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = 0.3f + threadIdx.x * 1e-6f + c * 1e-3f;
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = sinf_a(x[c]) + cosf_a(x[c]) * 0.5f;
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c];
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
 __device__ __forceinline__ float lg2f(float x) { float y; asm volatile("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
 __device__ __forceinline__ float rcpf(float x) { float y; asm volatile("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x)); return y; }
 __global__ void k_lg2(float* out, float a, float b, int iters) {
@@ -260,6 +292,7 @@ int main() {
         {"mufu_rsq", k_rsq, CH}, {"mufu_ex2(+fmul)", k_ex2, CH},
         {"ffma2_3reg_pairs", k_ffma2_3reg, 2.0 * CH},
         {"mufu_lg2(+fadd)", k_lg2, CH}, {"mufu_rcp", k_rcp, CH},
+        {"mufu_sin(+fmul.rz)", k_sin, CH}, {"mufu_sin+cos(+2 fmul.rz, ffma)", k_sincos, 2.0 * CH},
         {"dfma(fp64 lanes)", k_dfma, CH}, {"ffma2+dfma(fp32 lanes only)", k_mix, 2.0 * CH},
         {"f32->f64->f32 roundtrips(+dmul)", k_f2d, CH},
     };
