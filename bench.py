@@ -471,6 +471,89 @@ def cpu_oracle_sample(n: int, targets: int):
     return targets * float(n) / dt, dt
 
 
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+class one_core:
+    """Pin this process to one host core while the oracle is timed (the oracle
+    beside the GPU runs single-threaded on one pinned core)."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0) if hasattr(os, "sched_getaffinity") else None
+        if self.old:
+            os.sched_setaffinity(0, {min(self.old)})
+        return self
+
+    def __exit__(self, *exc):
+        if self.old:
+            os.sched_setaffinity(0, self.old)
+
+
+def oracle_beside(configs: dict) -> None:
+    """Time the oracle (as it stands, one pinned core) on a bounded sample of every config's
+    workload and attach it as configs[k]["cpu_oracle"] in the config's own unit."""
+    import oracle
+    oracle.lib()
+
+    def timed(fn):
+        t = time.perf_counter()
+        r = fn()
+        return r, time.perf_counter() - t
+
+    def put(key, units, secs, sample):
+        if key in configs and isinstance(configs[key], dict):
+            configs[key]["cpu_oracle"] = {"value": units / secs, "unit": configs[key].get("unit"), "cores": 1,
+                                          "kind": "oracle", "sample": f"{sample} ({secs:.2f} s)"}
+
+    with one_core():
+        b = inputs.nbody_bodies(4096, seed=1)
+        _, sec = timed(lambda: oracle.nbody_accel(b, np.float32(EPS2)))
+        put("nbody_4096", 4096.0 * 4096, sec, "full 4096 x 4096 force map")
+        put("nbody_4096_graph", 4096.0 * 4096, sec, "one 4096 x 4096 force map (integrator negligible)")
+        put("nbody_4096_simulate", 4096.0 * 4096, sec, "one 4096 x 4096 force map (integrator negligible)")
+        S, X, T = inputs.blackscholes_options(1 << 20, seed=2)
+        _, sec = timed(lambda: oracle.blackscholes(S, X, T, inputs.BS_R, inputs.BS_SIGMA))
+        put("blackscholes_map", float(1 << 20), sec, "2^20 of the 2^24 options")
+        _, sec = timed(lambda: oracle.blackscholes_sums(S, X, T, inputs.BS_R, inputs.BS_SIGMA))
+        put("blackscholes_map_reduce", float(1 << 20), sec, "2^20 of the 2^24 options")
+        W = 8192
+        rows = 64
+        _, sec = timed(lambda: oracle.mandelbrot(W, W, 0, W // rows, rows, -2.0, -1.5, 3.0 / W, 3.0 / W, 1024))
+        put("mandelbrot", float(rows * W), sec, f"{rows} rows spread evenly over the 8192^2 frame")
+        A = inputs.bf16_uniform(64, 8192, 4, 0)
+        Bt = inputs.bf16_uniform(64, 8192, 4, 1)
+        rr = np.random.default_rng(0).integers(0, 64, size=(2, 8192))
+        _, sec = timed(lambda: oracle.matmul_bf16_entries(A, Bt, rr[0], rr[1]))
+        put("matmul", 8192.0, sec, "8192 dot products of length K = 8192")
+        b64 = inputs.nbody_bodies(1 << 20, seed=5).astype(np.float64)
+        _, sec = timed(lambda: oracle.nbody_accel_f64(b64, 1e-4, 0, 32))
+        put("nbody_f64", 32.0 * (1 << 20), sec, "32 targets x 2^20 sources")
+        atoms = inputs.cp_atoms()
+        _, sec = timed(lambda: oracle.coulomb_potential(atoms, inputs.CP_NX, 8, inputs.CP_Z, inputs.CP_H))
+        put("parboil_cp", 8.0 * inputs.CP_NX * atoms.shape[0], sec, "8 lattice rows x all atoms")
+        ks, vx = inputs.mriq_kspace(), inputs.mriq_voxels()
+        _, sec = timed(lambda: oracle.mriq(ks, vx[:2048]))
+        put("parboil_mriq", 2048.0 * ks.shape[0], sec, "2048 voxels x all k-samples")
+        _, sec = timed(lambda: oracle.series(0, 1000))
+        put("jg_series_f32", 1000.0, sec, "coefficients 0..999")
+        put("jg_series_f64", 1000.0, sec, "coefficients 0..999")
+        data = inputs.crypt_data()
+        ek, _ = oracle.idea_keys(inputs.crypt_key())
+        _, sec = timed(lambda: oracle.idea(data, ek))
+        put("jg_crypt", float(data.shape[0]), sec, "the full 3 MiB")
+        x = np.ones(1 << 26, dtype=np.float32)
+        _, sec = timed(lambda: oracle.reduce("sum", x, "f32"))
+        put("reduce_sum_f32", float(1 << 26), sec, "2^26 of the 2^28 elements")
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return None
@@ -529,10 +612,13 @@ def main():
             props = torch.cuda.get_device_properties(local)
             flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
             line["configs"] = run_extras(peaks, flush)
-        v, secs = cpu_oracle_sample(args.n, args.cpu_targets)
+            oracle_beside(line["configs"])
+        with one_core():
+            v, secs = cpu_oracle_sample(args.n, args.cpu_targets)
         line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"{args.cpu_targets} targets x {args.n} sources of step 0 "
-                                          f"({secs:.1f} s, single-threaded C fp64)"}
+                                          f"({secs:.1f} s, single-threaded C fp64, one pinned core)",
+                                "host_cpu": cpu_model(), "host_cores": os.cpu_count()}
     elif rank == 0:
         line["cpu_baseline"] = None
     line["peaks"] = peaks
