@@ -229,3 +229,36 @@ def test_simulate_host_small_path(lime):
     pos, vel = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
     _eager_steps(lime, pos, vel, steps)
     assert torch.equal(h_pos, pos.cpu()) and torch.equal(h_vel, vel.cpu())
+
+
+def test_config5_steps_one_step_parity(lime):
+    # SURVEY.md §8(c) C-integrator: at each checked step the oracle recomputes the forces of sampled
+    # targets against all 2^20 sources FROM THE GPU'S CURRENT POSITIONS and applies the integrator
+    # (one-step parity; avoids comparing chaotic multi-step trajectories).
+    n, steps, dt = 1 << 20, 3, 1e-3
+    b = inputs.nbody_bodies(n, seed=5)
+    pos, vel = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    rows = np.concatenate([np.random.default_rng(3).choice(n, 96, replace=False), [0, n - 1]])
+    for _ in range(steps):
+        p0, v0 = pos.cpu().numpy(), vel.cpu().numpy()
+        lime.nbody_simulate(pos, vel, 1, float(EPS2), dt)
+        acc, mag = oracle.nbody_accel_rows(p0, EPS2, rows, threads=8)
+        a4 = np.zeros((rows.size, 4), np.float32)
+        a4[:, :3] = acc
+        po, vo = oracle.nbody_integrate(p0[rows], v0[rows], a4, np.float32(dt))
+        vg, pg = vel.cpu().numpy()[rows], pos.cpu().numpy()[rows]
+        dv = np.abs(vg[:, :3] - vo[:, :3]).max(axis=1)
+        assert (dv <= NBODY_RTOL * mag * dt + 4e-7 * np.abs(vo[:, :3]).max(axis=1) + 1e-12).all(), dv.max()
+        np.testing.assert_allclose(pg, po, rtol=0, atol=3e-7)
+
+
+def test_momentum_after_ten_steps(lime):
+    # SURVEY.md §8(c) pin: |sum m v| <= 1e-6 sum m |v| after 10 steps from rest
+    for n in (4096, 1 << 16):
+        b = inputs.nbody_bodies(n, seed=11)
+        pos, vel = _dev(b), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+        lime.nbody_simulate(pos, vel, 10, float(EPS2), 1e-3)
+        m = b[:, 3].astype(np.float64)
+        v = vel.cpu().numpy()[:, :3].astype(np.float64)
+        P = (m[:, None] * v).sum(0)
+        assert np.linalg.norm(P) <= 1e-6 * (m * np.linalg.norm(v, axis=1)).sum()
