@@ -51,6 +51,53 @@ __global__ void k_ffma2(float* out, float a, float b, int iters) {
     if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
 }
 
+// FFMA2 whose scalar operands are compile-time constants (ptxas encodes them as immediates)
+__global__ void k_ffma2_imm(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float2 x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = make_float2(threadIdx.x * 1e-3f + c, c);
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = ffma2(x[c], make_float2(0.999f, 0.999f), make_float2(1e-3f, 1e-3f));
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c].x + x[c].y;
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+// FFMA2 with one 32-bit register broadcast operand (.F32) and one pair
+__global__ void k_ffma2_bcast(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float2 x[CH];
+    float av = a + threadIdx.x * 1e-9f;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = make_float2(threadIdx.x * 1e-3f + c, c);
+    const float2 B = make_float2(b + threadIdx.x * 1e-9f, b);
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = ffma2(x[c], make_float2(av, av), B);
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c].x + x[c].y;
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
+// FADD2 with an immediate (the 1.5*2^23 rounding trick)
+__global__ void k_fadd2_imm(float* out, float a, float b, int iters) {
+    long long t0 = clock64();
+    float2 x[CH];
+#pragma unroll
+    for (int c = 0; c < CH; ++c) x[c] = make_float2(threadIdx.x * 1e-3f + c, c);
+    for (int i = 0; i < iters; ++i)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) x[c] = fadd2(x[c], make_float2(1e-3f, 1e-3f));
+    float s = 0;
+#pragma unroll
+    for (int c = 0; c < CH; ++c) s += x[c].x + x[c].y;
+    if (s == 12345.f) out[0] = s;
+    if (threadIdx.x == 0) g_cycles[blockIdx.x] = clock64() - t0;
+}
 __global__ void k_fadd2(float* out, float a, float b, int iters) {
     long long t0 = clock64();
     float2 x[CH];
@@ -289,6 +336,8 @@ int main() {
     const int threads = 256, blocks = sms * 4, iters = 1 << 14;
     struct { const char* name; void (*k)(float*, float, float, int); double lane_ops_per_iter; } tests[] = {
         {"ffma", k_ffma, CH}, {"ffma2", k_ffma2, 2.0 * CH}, {"fadd2", k_fadd2, 2.0 * CH},
+        {"ffma2_imm", k_ffma2_imm, 2.0 * CH}, {"ffma2_bcast_reg", k_ffma2_bcast, 2.0 * CH},
+        {"fadd2_imm", k_fadd2_imm, 2.0 * CH},
         {"mufu_rsq", k_rsq, CH}, {"mufu_ex2(+fmul)", k_ex2, CH},
         {"ffma2_3reg_pairs", k_ffma2_3reg, 2.0 * CH},
         {"mufu_lg2(+fadd)", k_lg2, CH}, {"mufu_rcp", k_rcp, CH},
