@@ -47,6 +47,13 @@ def main(which):
         b = torch.from_numpy(inputs.nbody_bodies(n, seed=1)).cuda()
         acc = torch.empty_like(b)
         out["nbody4096_us"] = 1e3 * time_launches(lambda: lime.map_nbody(b, 1e-4, out=acc), 50, 5, flush)[0]
+    if "nbody1m" in which:
+        n = 1 << 20
+        b = torch.from_numpy(inputs.nbody_bodies(n, seed=5)).cuda()
+        acc = torch.empty_like(b)
+        ms = time_launches(lambda: lime.map_nbody(b, 1e-4, out=acc), 3, 1, flush)[0]
+        out["nbody1m_ms"] = ms
+        out["nbody1m_frac"] = 20.0 * n * n / (ms * 1e-3) / 74.45e12
     if "nbody64" in which:
         for n, cnt in ((4096, 4096), (1 << 20, 1 << 17)):
             b = torch.from_numpy(inputs.nbody_bodies(n, seed=1).astype(np.float64)).cuda()
