@@ -12,7 +12,7 @@ from ncu_summary import summarize  # noqa: E402
 KEYMAP = {"nbody1m": "nbody_force_1m", "nbody1m_p8": "nbody_force_1m_p8", "nbody4096": "nbody_force_4096",
           "bs_map": "bs_map", "bs_fused": "bs_map_reduce", "mandel": "mandelbrot", "matmul": "matmul",
           "reduce": "reduce_sum_f32", "cp": "parboil_cp", "mriq": "parboil_mriq",
-          "nbody64": "nbody_f64", "series": "jg_series_f32", "idea": "jg_crypt"}
+          "nbody64": "nbody_f64", "series": "jg_series_f32", "idea": "jg_crypt", "sim4096": "nbody_simulate_4096"}
 
 
 def main(tag):

@@ -3,7 +3,7 @@
     ncu --set full --clock-control none --import-source on -k regex:<kernel> -s 1 -c 1 \
         -o gpurun_out/prof_<which> python tools/prof_kernels.py <which>
 
-which: nbody1m | nbody1m_p8 | nbody4096 | nbody64 | bs_map | bs_fused | mandel | matmul | reduce | cp | mriq
+which: nbody1m | nbody1m_p8 | nbody4096 | sim4096 | nbody64 | bs_map | bs_fused | mandel | matmul | reduce | cp | mriq
        | series | idea
 """
 import os
@@ -19,7 +19,7 @@ from paper_conf_pldi_dubachcrbf12_b200 import inputs  # noqa: E402
 
 def main(which: str, reps: int = 3):
     lime.load()
-    if which.startswith("nbody"):
+    if which.startswith("nbody") and which != "nbody64":
         n = 4096 if which == "nbody4096" else 1 << 20
         b = torch.from_numpy(inputs.nbody_bodies(n, seed=5)).cuda()
         cnt = n // 8 if which.endswith("_p8") else n
@@ -53,6 +53,11 @@ def main(which: str, reps: int = 3):
         vx = torch.from_numpy(inputs.mriq_voxels()).cuda()
         for _ in range(reps):
             lime.map_mriq(k, vx)
+    elif which == "sim4096":
+        p = torch.from_numpy(inputs.nbody_bodies(4096, seed=1)).cuda()
+        v = torch.zeros_like(p)
+        for _ in range(reps):
+            lime.nbody_simulate(p, v, 100, 1e-4, 1e-3)
     elif which == "nbody64":
         b = torch.from_numpy(inputs.nbody_bodies(1 << 20, seed=5).astype(np.float64)).cuda()
         for _ in range(reps):
