@@ -96,8 +96,9 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
  *   eps2    Plummer softening, finite and > 0 (eps2 <= 0 makes the self term 0/0).
  *   0 <= tgt_begin, 0 <= tgt_count, tgt_begin + tgt_count <= n_src.
  * Summation order (deterministic, independent of launch config and of the
- * target shard): sources are cut into 256-body chunks; each chunk is summed in
- * j order into a chunk partial; chunk partials are added in order into one of
+ * target shard): sources are cut into chunks (128 bodies when n_src <= 8192,
+ * else 256); each chunk is summed in j order into a chunk partial; chunk
+ * partials are added in order into one of
  * S = nbody_splits(n_src) split partials; split partials are added in s order.
  * Launch override: grid ignored; block_threads in {128, 256}; per_thread in {1, 2, 4, 8}.
  * =========================================================================== */

@@ -18,10 +18,21 @@ int device_num_sms();
 
 // ------------------------------------------------------------------ N-Body
 namespace nbody {
-constexpr int kChunk = 256;      // two-level accumulation chunk (part of the result's definition)
-constexpr int kMaxSplits = 16;   // split-j partials per target (function of n_src only)
+// Two-level accumulation (part of the result's definition, a function of n_src only): sources are
+// cut into chunks of chunk_len(n_src) bodies whose partials are added in order into one of
+// splits(n_src) split partials, added in split order. Small problems (n_src <= kSmallMaxSources)
+// use 128-body chunks and up to 32 splits (twice the warps for the latency-bound sizes), larger
+// ones 256-body chunks and up to 16 splits.
+constexpr int kChunk = 256;
+constexpr int kMaxSplits = 16;
+constexpr int kChunkSmall = 128;
+constexpr int kMaxSplitsSmall = 32;
+constexpr int64_t kSmallMaxSources = 8192;
+int chunk_len(int64_t n_src);
 int64_t chunks_per_split(int64_t n_src);
 int splits(int64_t n_src);
+int64_t chunks_per_split_fixed(int64_t n_src);   // 256-body chunks, <= 16 splits (fp64 map)
+int splits_fixed(int64_t n_src);
 size_t workspace_bytes(int64_t n_src, int64_t tgt_count);
 cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,
                          float eps2, float4* accel, void* ws, cudaStream_t stream);

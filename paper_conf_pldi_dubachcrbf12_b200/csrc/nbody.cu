@@ -15,7 +15,7 @@
 //    packed FADD2/FFMA2/FMUL2 (6 issue slots per interaction); bit-identical to the scalar
 //    variant (each half is one IEEE op in the same order).
 //  * A1 (L201-208): results are independent of the launch configuration: a target's sum
-//    order is fixed by the 256-body chunk grid and the split count, both functions of n_src.
+//    order is fixed by the chunk grid (128 or 256 bodies) and the split count, both functions of n_src.
 //  * A8 (split-j): S = splits(n_src) source ranges are processed by separate CTAs; the last
 //    CTA of a target tile to finish (atomic ticket) adds the S partials in s order --
 //    one launch, deterministic, self-resetting counters.
@@ -26,17 +26,23 @@ namespace lime {
 namespace nbody {
 
 constexpr int kTileJ = 1024;   // sources per shared-memory stage (16 KB)
-static_assert(kTileJ % kChunk == 0, "stage must hold whole chunks");
+static_assert(kTileJ % kChunk == 0 && kTileJ % kChunkSmall == 0, "stage must hold whole chunks");
 
-int64_t chunks_per_split(int64_t n_src) {
-    const int64_t chunks = ceil_div<int64_t>(n_src, kChunk);
-    return chunks == 0 ? 1 : ceil_div<int64_t>(chunks, kMaxSplits);
+int chunk_len(int64_t n_src) { return n_src <= kSmallMaxSources ? kChunkSmall : kChunk; }
+static int max_splits(int64_t n_src) { return n_src <= kSmallMaxSources ? kMaxSplitsSmall : kMaxSplits; }
+static int64_t cps_rule(int64_t n_src, int chunk, int maxs) {
+    const int64_t chunks = ceil_div<int64_t>(n_src, chunk);
+    return chunks == 0 ? 1 : ceil_div<int64_t>(chunks, maxs);
 }
-int splits(int64_t n_src) {
-    const int64_t chunks = ceil_div<int64_t>(n_src, kChunk);
+static int splits_rule(int64_t n_src, int chunk, int maxs) {
+    const int64_t chunks = ceil_div<int64_t>(n_src, chunk);
     if (chunks <= 1) return 1;
-    return static_cast<int>(ceil_div<int64_t>(chunks, chunks_per_split(n_src)));
+    return static_cast<int>(ceil_div<int64_t>(chunks, cps_rule(n_src, chunk, maxs)));
 }
+int64_t chunks_per_split(int64_t n_src) { return cps_rule(n_src, chunk_len(n_src), max_splits(n_src)); }
+int splits(int64_t n_src) { return splits_rule(n_src, chunk_len(n_src), max_splits(n_src)); }
+int64_t chunks_per_split_fixed(int64_t n_src) { return cps_rule(n_src, kChunk, kMaxSplits); }
+int splits_fixed(int64_t n_src) { return splits_rule(n_src, kChunk, kMaxSplits); }
 
 // workspace: [counters: one u32 per 128-target tile, padded to 256 B][partials: S x count float4]
 static size_t counters_bytes(int64_t tgt_count) {
@@ -58,7 +64,8 @@ struct ForceArgs {
     float4* partial;      // [S][tgt_count]
     unsigned* counters;   // [tiles]
     int splits;
-    int64_t split_len;    // chunks_per_split * kChunk
+    int chunk;            // chunk_len(n_src)
+    int64_t split_len;    // chunks_per_split * chunk
 };
 
 template <int R, bool kPacked>
@@ -206,7 +213,7 @@ __device__ __forceinline__ void finish_targets(const ForceArgs& a, const IT& it,
     if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
 }
 
-template <int BLOCK, int R, bool kPacked>
+template <int BLOCK, int R, bool kPacked, int CHUNK>
 __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ ForceArgs a) {
     __shared__ __align__(128) float4 sbuf[2][kTileJ];
     __shared__ __align__(8) uint64_t full[2];
@@ -255,12 +262,12 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
         mbar_wait(&full[t & 1], (t >> 1) & 1);
         const float4* sb = sbuf[t & 1];
         const int len = static_cast<int>(mn<int64_t>(kTileJ, j1 - (j0 + static_cast<int64_t>(t) * kTileJ)));
-        for (int c0 = 0; c0 < len; c0 += kChunk) {
-            const int c1 = min(len, c0 + kChunk);
+        for (int c0 = 0; c0 < len; c0 += CHUNK) {
+            const int c1 = min(len, c0 + CHUNK);
             it.chunk_begin();
-            if (c1 - c0 == kChunk) {
+            if (c1 - c0 == CHUNK) {
 #pragma unroll 4
-                for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
+                for (int j = c0; j < c0 + CHUNK; ++j) it.body(sb[j], eps2);
             } else {
                 for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
             }
@@ -282,16 +289,17 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
 // shared memory. Same summation order as force_kernel, hence bit-identical results, but no global
 // partials, no atomic tickets and ~16 warps per SM instead of 1-2 CTAs of 4 warps.
 // =====================================================================================
-constexpr int64_t kSmallMaxSources = 8192;
-
 // One split's contribution for one target: chunk partials added into the split accumulator in chunk
 // order -- the arithmetic of force_kernel's scalar variant (shared by force_small_kernel and the
 // persistent simulation kernel, so all three agree bit for bit).
-__device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* sb, int len, float eps2) {
-    for (int c0 = 0; c0 < len; c0 += kChunk) {
-        const int c1 = mn(len, c0 + kChunk);
+__device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* sb, int len, int chunk, float eps2) {
+    for (int c0 = 0; c0 < len; c0 += chunk) {
+        const int c1 = mn(len, c0 + chunk);
         it.chunk_begin();
-        if (c1 - c0 == kChunk) {
+        if (c1 - c0 == kChunkSmall) {
+#pragma unroll 4
+            for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
+        } else if (c1 - c0 == kChunk) {
 #pragma unroll 4
             for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
         } else {
@@ -301,11 +309,11 @@ __device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* 
     }
 }
 
-__global__ void __launch_bounds__(32 * kMaxSplits) force_small_kernel(const __grid_constant__ ForceArgs a) {
+__global__ void __launch_bounds__(32 * kMaxSplitsSmall) force_small_kernel(const __grid_constant__ ForceArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                          // [S][split_len]
     float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
-    __shared__ __align__(8) uint64_t bar[kMaxSplits];
+    __shared__ __align__(8) uint64_t bar[kMaxSplitsSmall];
 
     const int warp = threadIdx.x >> 5;            // = split index
     const unsigned lane = lane_id();
@@ -327,7 +335,7 @@ __global__ void __launch_bounds__(32 * kMaxSplits) force_small_kernel(const __gr
     }
     __syncwarp();
     mbar_wait(&bar[warp], 0);
-    split_sum(it, sb, len, a.eps2);
+    split_sum(it, sb, len, a.chunk, a.eps2);
     part[warp * 32 + lane] = it.result(0);
     __syncthreads();
     if (warp == 0 && valid) {
@@ -346,9 +354,9 @@ static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
     static size_t attr = 0;
     if (smem > attr) {
         cudaError_t e = cudaFuncSetAttribute(force_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplits * 32 * 16));
+                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
         if (e != cudaSuccess) return e;
-        attr = kSmallMaxSources * 16 + kMaxSplits * 32 * 16;
+        attr = kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16;
     }
     const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
     force_small_kernel<<<static_cast<unsigned>(ctas), 32 * a.splits, smem, stream>>>(a);
@@ -378,6 +386,7 @@ struct SimArgs {
     int64_t n;
     int32_t steps;
     int32_t splits;
+    int32_t chunk;
     int64_t split_len;
     float eps2, dt;
 };
@@ -395,7 +404,7 @@ __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(32 * kMaxSplits) simulate_small_kernel(const __grid_constant__ SimArgs a) {
+__global__ void __launch_bounds__(32 * kMaxSplitsSmall) simulate_small_kernel(const __grid_constant__ SimArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                                   // [S][split_len]
     float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
@@ -419,7 +428,7 @@ __global__ void __launch_bounds__(32 * kMaxSplits) simulate_small_kernel(const _
             Interact<1, false> it;
             it.set(0, p);
             it.zero_all();
-            split_sum(it, sb, len, a.eps2);
+            split_sum(it, sb, len, a.chunk, a.eps2);
             part[warp * 32 + lane] = it.result(0);
             __syncthreads();
             if (warp == 0 && valid) {
@@ -490,7 +499,8 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.n = n;
     a.steps = steps;
     a.splits = splits(n);
-    a.split_len = chunks_per_split(n) * kChunk;
+    a.chunk = chunk_len(n);
+    a.split_len = chunks_per_split(n) * a.chunk;
     a.eps2 = eps2;
     a.dt = dt;
     const int block = 32 * a.splits;
@@ -498,7 +508,7 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(simulate_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplits * 32 * 16));
+                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
         if (e != cudaSuccess) return e;
         attr = true;
     }
@@ -589,12 +599,15 @@ __global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_consta
             else if constexpr (V == 5) return tile4[j];
             else return c_bodies[g];
         };
-        for (int c0 = 0; c0 < len; c0 += kChunk) {
-            const int c1 = mn(len, c0 + kChunk);
+        for (int c0 = 0; c0 < len; c0 += a.chunk) {
+            const int c1 = mn(len, c0 + a.chunk);
             it.chunk_begin();
             if (c1 - c0 == kChunk) {
 #pragma unroll 4
                 for (int j = c0; j < c0 + kChunk; ++j) it.body(src(j), eps2);
+            } else if (c1 - c0 == kChunkSmall) {
+#pragma unroll 4
+                for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(src(j), eps2);
             } else {
                 for (int j = c0; j < c1; ++j) it.body(src(j), eps2);
             }
@@ -632,7 +645,8 @@ static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
     const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
     dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
-    force_kernel<BLOCK, R, kPacked><<<grid, BLOCK, 0, stream>>>(a);
+    if (a.chunk == kChunk) force_kernel<BLOCK, R, kPacked, kChunk><<<grid, BLOCK, 0, stream>>>(a);
+    else force_kernel<BLOCK, R, kPacked, kChunkSmall><<<grid, BLOCK, 0, stream>>>(a);
     return cudaGetLastError();
 }
 
@@ -647,7 +661,8 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.eps2 = eps2;
     a.accel = accel;
     a.splits = splits(n_src);
-    a.split_len = chunks_per_split(n_src) * kChunk;
+    a.chunk = chunk_len(n_src);
+    a.split_len = chunks_per_split(n_src) * a.chunk;
     a.counters = static_cast<unsigned*>(ws);
     a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
 

@@ -33,7 +33,7 @@ static size_t counters_bytes(int64_t tgt_count) {
     return ((ceil_div<int64_t>(tgt_count, kBlock * kR) * 4 + 255) / 256) * 256;
 }
 size_t workspace_bytes(int64_t n_src, int64_t tgt_count) {
-    const int S = nbody::splits(n_src);
+    const int S = nbody::splits_fixed(n_src);
     return counters_bytes(tgt_count) + (S > 1 ? static_cast<size_t>(S) * tgt_count * 32 : 0) + 256;
 }
 
@@ -161,8 +161,8 @@ cudaError_t launch_force(const double* bodies, int64_t n_src, int64_t tgt_begin,
     a.tgt_count = tgt_count;
     a.eps2 = eps2;
     a.accel = reinterpret_cast<double4*>(accel);
-    a.splits = nbody::splits(n_src);
-    a.split_len = nbody::chunks_per_split(n_src) * nbody::kChunk;
+    a.splits = nbody::splits_fixed(n_src);
+    a.split_len = nbody::chunks_per_split_fixed(n_src) * nbody::kChunk;
     a.counters = static_cast<unsigned*>(ws);
     a.partial = reinterpret_cast<double4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
     const int64_t tiles = ceil_div<int64_t>(tgt_count, static_cast<int64_t>(kBlock) * kR);

@@ -125,9 +125,12 @@ def test_no_device_reports_unsupported(L):
 
 def test_workspace_queries_and_split_rule(L):
     # splits depend on n_src only (deterministic order across shards/launches)
-    assert L.lime_nbody_splits(1) == 1 and L.lime_nbody_splits(256) == 1
-    assert L.lime_nbody_splits(257) == 2
-    assert L.lime_nbody_splits(4096) == 16
+    # n_src <= 8192: 128-body chunks, <= 32 splits; larger: 256-body chunks, <= 16 splits
+    assert L.lime_nbody_splits(1) == 1 and L.lime_nbody_splits(128) == 1
+    assert L.lime_nbody_splits(129) == 2 and L.lime_nbody_splits(257) == 3
+    assert L.lime_nbody_splits(4096) == 32
+    assert L.lime_nbody_splits(8192) == 32          # 64 chunks, 2 per split
+    assert L.lime_nbody_splits(8193) == 11          # 33 chunks of 256, 3 per split
     assert L.lime_nbody_splits(1 << 20) == 16
     assert L.lime_map_nbody_workspace_bytes(1 << 20, 1 << 17) >= 16 * (1 << 17) * 16
     assert L.lime_reduce_workspace_bytes() >= 256
