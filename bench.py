@@ -39,6 +39,9 @@ UNIT = "interactions/s"
 EPS2, DT = 1e-4, 1e-3
 FLOP_PER_INTERACTION = 20          # GPU Gems 3 convention
 FP32_LANE_OPS_PER_INTERACTION = 12  # 3 FADD + 3 FFMA (r^2) + 3 FMUL + 3 FFMA (acc)
+# mass-uniform splits (R11; the equal-mass workload): the mass factors out of each chunk
+# sum, 2 FMUL instead of 3 -> 11 FP32 lane-ops per interaction (the 20-flop convention is unchanged)
+FP32_LANE_OPS_UNIFORM_MASS = 11
 SM_MAX_MHZ_NOMINAL = 1965.0
 SMS_B200 = 148
 
@@ -133,16 +136,39 @@ def flush_l2(buf):
     buf.fill_(1)   # write > L2 (2x l2CacheSize) so the next launch starts cold
 
 
+_CLEAN = {}
+
+
+def flush_l2_clean(buf):
+    """Write > L2 (the contract's flush), then read a second buffer > L2 so the dirty lines the
+    write left behind are written back BEFORE the timed launch (tools/hbm_probe.cu measured the
+    write-back of a write-only flush at ~4 us inside a 35-us streaming kernel,
+    profiles/experiments/hbm_probe_r01.jsonl); the L2 then holds clean lines of an unrelated buffer."""
+    buf.fill_(1)
+    key = (buf.device, buf.numel())
+    if key not in _CLEAN:
+        _CLEAN[key] = torch.zeros(buf.numel() // 4, dtype=torch.int32, device=buf.device)
+    torch.amax(_CLEAN[key])
+
+
+# GPU-side idle before each timed launch: while the device sleeps the host enqueues the start
+# event and the launch, so host-side Python/ctypes time never lands between the two events
+# (~100 us at 1.9 GHz; outside the event pair).
+SLEEP_CYCLES = 200_000
+
+
 def time_launches(fn, iters, warmup, flush_buf=None):
     """Median/mean device time of `fn` over `iters` launches, each bracketed by CUDA events on the
-    current stream; the L2 is flushed before every launch (outside the event pair)."""
+    current stream; the L2 is flushed (write, then a clean read) before every launch, outside the
+    event pair, followed by a short device sleep so the launch is queued before the start event."""
     for _ in range(warmup):
         fn()
     torch.cuda.synchronize()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(iters)]
     for a, b in ev:
         if flush_buf is not None:
-            flush_l2(flush_buf)
+            flush_l2_clean(flush_buf)
+        torch.cuda._sleep(SLEEP_CYCLES)
         a.record()
         fn()
         b.record()
@@ -232,11 +258,19 @@ def run_nbody(args, rank, world, local):
     per_launch_interactions = float(sim.count) * n
     achieved = FLOP_PER_INTERACTION * per_launch_interactions / (force_ms * 1e-3) / 1e12
     obs_mhz = clk.get("sm_mhz") or SM_MAX_MHZ_NOMINAL
-    pipe_frac = (FP32_LANE_OPS_PER_INTERACTION * per_launch_interactions / (force_ms * 1e-3)) / (SMS_B200 * 128 * obs_mhz * 1e6)
+    uniform_mass = bool(torch.all(bodies[:, 3] == bodies[0, 3]).item())
+    lane_ops = FP32_LANE_OPS_UNIFORM_MASS if uniform_mass else FP32_LANE_OPS_PER_INTERACTION
+    pipe_frac = (lane_ops * per_launch_interactions / (force_ms * 1e-3)) / (SMS_B200 * 128 * obs_mhz * 1e6)
     roofline = {"kernel": "lime::nbody::force_kernel", "bound": "alu", "achieved": achieved, "peak": peak,
                 "unit": "TFLOP/s", "frac": achieved / peak, "traffic": ncu_traffic("nbody_force_1m"),
                 "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 flop x 1965 MHz (microbench: 124.9-127.9 lane-ops/clk/SM)",
                 "flop_per_interaction": FLOP_PER_INTERACTION,
+                "fp32_lane_ops_per_interaction": lane_ops,
+                "element_form": "mass factored out of each chunk sum (equal masses, DESIGN.md R11)" if uniform_mass
+                                else "per-body mass multiply",
+                "fp32_lane_ops_per_interaction": lane_ops,
+                "element_form": ("mass factored out of each chunk sum (equal masses, DESIGN.md R11)" if uniform_mass
+                                 else "per-body mass multiply"),
                 "fp32_pipe_frac_at_observed_clock": pipe_frac, "observed_sm_mhz": obs_mhz,
                 "force_ms_per_launch": force_ms, "force_ms_per_launch_max_rank": force_ms_max,
                 "force_share_of_step": force_ms / (ms_local / args.steps)}
@@ -250,7 +284,7 @@ def run_nbody(args, rank, world, local):
                        "l2": "flushed before every step inside the timed region (2x L2 write); the 16 MiB source "
                              "array is then re-read from L2 by design (broadcast operand)",
                        "inputs": "inputs.nbody_bodies(seed=5): U[-1,1)^3, m=1/N, v0=0"},
-            "roofline": roofline, "e2e": e2e, "gpu_launches": 2 * args.steps, "clocks": clk,
+            "roofline": roofline, "e2e": e2e, "gpu_launches": (4 if n > 8192 else 2) * args.steps + (args.steps if world > 1 else 0), "clocks": clk,
             "momentum_residual": float(mom.norm().item())}
     return line
 
@@ -377,6 +411,29 @@ def run_extras(peaks, flush):
         del A, Bt, Cm
     except lime.LimeError as e:
         out["matmul"] = {"workload": "configs[3]", "unavailable": str(e)}
+
+    # config 5 per-GPU shard at P = 8 (2^17 targets x 2^20 sources): the workload's equal masses take
+    # the mass-factored element (11 FP32 lane-ops, R11); the same bodies with unequal
+    # masses (U[0.5, 1.5)/N) take the per-body-mass element (12) -- both reported
+    b1m = inputs.nbody_bodies(1 << 20, seed=5)
+    b1m_mixed = b1m.copy()
+    b1m_mixed[:, 3] = ((0.5 + inputs.uniform24(5, 99, 1 << 20)) / (1 << 20)).astype(np.float32)
+    acc1m = torch.empty((1 << 17, 4), dtype=torch.float32, device="cuda")
+    inter = float(1 << 20) * (1 << 17)
+    for key, arr, ops in (("nbody_1m_p8_shard", b1m, FP32_LANE_OPS_UNIFORM_MASS),
+                          ("nbody_1m_p8_shard_mixed_masses", b1m_mixed, FP32_LANE_OPS_PER_INTERACTION)):
+        bd = torch.from_numpy(arr).cuda()
+        med, _ = time_launches(lambda: lime.map_nbody(bd, EPS2, 0, 1 << 17, out=acc1m), 3, 1, flush)
+        ach = FLOP_PER_INTERACTION * inter / (med * 1e-3) / 1e12
+        out[key] = {"workload": "config-5 shard at P=8: 2^17 targets x 2^20 sources fp32"
+                                + (", masses U[0.5,1.5)/N" if ops == FP32_LANE_OPS_PER_INTERACTION else ", equal masses"),
+                    "value": inter / (med * 1e-3), "unit": "interactions/s", "ms_per_launch": med,
+                    "fp32_lane_ops_per_interaction": ops,
+                    "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s", "frac": ach / fp32,
+                                 "fp32_pipe_frac": ops * inter / (med * 1e-3) / (SMS_B200 * 128 * SM_MAX_MHZ_NOMINAL * 1e6),
+                                 "traffic": None}}
+        del bd
+    del acc1m
 
     # F3: double-precision N-Body (Table 3) at the config-5 per-GPU shape of P = 8; FP64-pipe
     # bound: 16 FP64 ops per interaction at 64 lanes/clk/SM (microbench: 58.9 measured)
@@ -612,6 +669,10 @@ def main():
             props = torch.cuda.get_device_properties(local)
             flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
             line["configs"] = run_extras(peaks, flush)
+            line["configs_timing"] = ("per config: warm-up launches, then each timed launch preceded (outside the "
+                                      "CUDA-event pair) by an L2 flush = write of 2x L2 + read of another 2x L2 "
+                                      "buffer (clean lines), and a ~100-us device sleep so the launch is queued "
+                                      "before the start event; median over launches")
             oracle_beside(line["configs"])
         with one_core():
             v, secs = cpu_oracle_sample(args.n, args.cpu_targets)

@@ -19,6 +19,8 @@
 //  * A8 (split-j): S = splits(n_src) source ranges are processed by separate CTAs; the last
 //    CTA of a target tile to finish (atomic ticket) adds the S partials in s order --
 //    one launch, deterministic, self-resetting counters.
+#include <type_traits>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -44,14 +46,22 @@ int splits(int64_t n_src) { return splits_rule(n_src, chunk_len(n_src), max_spli
 int64_t chunks_per_split_fixed(int64_t n_src) { return cps_rule(n_src, kChunk, kMaxSplits); }
 int splits_fixed(int64_t n_src) { return splits_rule(n_src, kChunk, kMaxSplits); }
 
-// workspace: [counters: one u32 per 128-target tile, padded to 256 B][partials: S x count float4]
+// workspace: [counters: one u32 per 128-target tile, padded to 256 B]
+//            [chunk flags: one byte per 256-body source chunk when n_src > kSmallMaxSources, padded to 256 B]
+//            [partials: S x count float4]
+// The counters are zero-invariant (every launch leaves them zero); the flags are rewritten by
+// every launch (prepass_kernel) before the force kernel reads them.
 static size_t counters_bytes(int64_t tgt_count) {
     return ((ceil_div<int64_t>(tgt_count, 128) * 4 + 255) / 256) * 256;
+}
+static bool uses_chunk_flags(int64_t n_src) { return n_src > kSmallMaxSources; }
+static size_t flags_bytes(int64_t n_src) {
+    return uses_chunk_flags(n_src) ? static_cast<size_t>((ceil_div<int64_t>(n_src, kChunk) + 255) / 256) * 256 : 0;
 }
 size_t workspace_bytes(int64_t n_src, int64_t tgt_count) {
     const int S = splits(n_src);
     if (S == 1) return 256;
-    return counters_bytes(tgt_count) + static_cast<size_t>(S) * static_cast<size_t>(tgt_count) * 16;
+    return counters_bytes(tgt_count) + flags_bytes(n_src) + static_cast<size_t>(S) * static_cast<size_t>(tgt_count) * 16;
 }
 
 struct ForceArgs {
@@ -63,6 +73,7 @@ struct ForceArgs {
     float4* accel;
     float4* partial;      // [S][tgt_count]
     unsigned* counters;   // [tiles]
+    const uint8_t* uniform;   // [ceil(n_src / kChunk)] chunk-uniform-mass flags, or null (n_src <= kSmallMaxSources)
     int splits;
     int chunk;            // chunk_len(n_src)
     int64_t split_len;    // chunks_per_split * chunk
@@ -104,6 +115,26 @@ struct Interact<R, false> {
             cy[r] = fmaf(s, dy, cy[r]);
             cz[r] = fmaf(s, dz, cz[r]);
         }
+    }
+    // Chunk-uniform mass (see prepass_kernel): the chunk partial is sum_j d / R^3 and the
+    // common mass multiplies it once at chunk end -- 11 FP32 lane-ops per interaction instead of 12.
+    __device__ __forceinline__ void body_unit(const float4 b, const float eps2) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const float dx = b.x - px[r];
+            const float dy = b.y - py[r];
+            const float dz = b.z - pz[r];
+            const float r2 = fmaf(dx, dx, fmaf(dy, dy, fmaf(dz, dz, eps2)));
+            const float inv = rsqrt_approx(r2);
+            const float s = (inv * inv) * inv;            // (r^2 + eps^2)^{-3/2}
+            cx[r] = fmaf(s, dx, cx[r]);
+            cy[r] = fmaf(s, dy, cy[r]);
+            cz[r] = fmaf(s, dz, cz[r]);
+        }
+    }
+    __device__ __forceinline__ void chunk_end_scaled(const float m) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) { ax[r] = fmaf(m, cx[r], ax[r]); ay[r] = fmaf(m, cy[r], ay[r]); az[r] = fmaf(m, cz[r], az[r]); }
     }
     __device__ __forceinline__ float4 result(int r) const { return make_float4(ax[r], ay[r], az[r], 0.f); }
 };
@@ -164,11 +195,85 @@ struct Interact<R, true> {
             cz[q] = fma2(t[q], dz[q], cz[q]);
         }
     }
+    // Chunk-uniform mass: 11 packed FP32 ops per target pair and source (see the scalar variant).
+    __device__ __forceinline__ void body_unit(const float4 b, const float eps2) {
+        const float2 e2 = bcast2(eps2);
+        float2 dx[Q], dy[Q], dz[Q], r2[Q], inv[Q], t[Q];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dz[q] = sub2(bcast2(b.z), pz[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dz[q], dz[q], e2);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dy[q] = sub2(bcast2(b.y), py[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dy[q], dy[q], r2[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) dx[q] = sub2(bcast2(b.x), px[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) r2[q] = fma2(dx[q], dx[q], r2[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) inv[q] = make_float2(rsqrt_approx(r2[q].x), rsqrt_approx(r2[q].y));
+#pragma unroll
+        for (int q = 0; q < Q; ++q) t[q] = mul2(inv[q], inv[q]);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) t[q] = mul2(t[q], inv[q]);             // s = (inv inv) inv
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+            cx[q] = fma2(t[q], dx[q], cx[q]);
+            cy[q] = fma2(t[q], dy[q], cy[q]);
+            cz[q] = fma2(t[q], dz[q], cz[q]);
+        }
+    }
+    __device__ __forceinline__ void chunk_end_scaled(const float m) {
+        const float2 m2 = bcast2(m);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) { ax[q] = fma2(m2, cx[q], ax[q]); ay[q] = fma2(m2, cy[q], ay[q]); az[q] = fma2(m2, cz[q], az[q]); }
+    }
     __device__ __forceinline__ float4 result(int r) const {
         const int q = r >> 1;
         return (r & 1) ? make_float4(ax[q].y, ay[q].y, az[q].y, 0.f) : make_float4(ax[q].x, ay[q].x, az[q].x, 0.f);
     }
 };
+
+// Mass-uniform splits (R11): when every source of a split carries the same mass m
+// (bitwise-equal floats, e.g. equal-mass particle sets), m factors out of each chunk sum exactly --
+// sum_j m d_j / R_j^3 = m * sum_j d_j / R_j^3 -- so the chunk partials are accumulated without the
+// per-interaction mass multiply (11 FP32 lane-ops instead of 12) and scaled once at chunk end.
+// Applies to n_src > kSmallMaxSources (the FP32-pipe-bound sizes). A prepass writes one flag per
+// 256-body chunk; a split is mass-uniform when all its chunks are. The decision depends only on
+// the source data and the split grid (a function of n_src), so target shards and launch
+// configurations stay bit-identical.
+// The same prepass zeroes this call's split tickets, so stale scratch left in a reused workspace by
+// a call with other sizes can never reach a ticket (flags == nullptr: tickets only).
+__global__ void __launch_bounds__(256) prepass_kernel(const float4* __restrict__ bodies, int64_t n_src,
+                                                      uint8_t* __restrict__ flags, unsigned* __restrict__ counters,
+                                                      int64_t ncounters) {
+    for (int64_t k = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; k < ncounters;
+         k += static_cast<int64_t>(gridDim.x) * blockDim.x)
+        counters[k] = 0u;
+    if (flags == nullptr) return;
+    const int64_t nchunks = ceil_div<int64_t>(n_src, kChunk);
+    const int64_t warps = static_cast<int64_t>(gridDim.x) * (blockDim.x >> 5);
+    for (int64_t c = blockIdx.x * static_cast<int64_t>(blockDim.x >> 5) + (threadIdx.x >> 5); c < nchunks; c += warps) {
+        const int64_t c0 = c * kChunk, c1 = mn<int64_t>(n_src, c0 + kChunk);
+        const float m0 = __ldg(&bodies[c0].w);
+        bool uni = true;
+        for (int64_t j = c0 + lane_id(); j < c1; j += 32) uni &= (__ldg(&bodies[j].w) == m0);
+        uni = __all_sync(0xffffffffu, uni);
+        if (lane_id() == 0) flags[c] = uni ? 1 : 0;
+    }
+}
+
+// True when every chunk of the split [j0, j1) is mass-uniform AND all chunks share one mass
+// (chunk c's first body against the split's first body). Every thread of the CTA must call it.
+template <int BLOCK>
+__device__ __forceinline__ bool split_mass_uniform(const float4* bodies, const uint8_t* flags, int64_t j0, int64_t j1) {
+    const float m0 = __ldg(&bodies[j0].w);
+    bool all = true;
+    for (int64_t c = j0 / kChunk + threadIdx.x; c < ceil_div<int64_t>(j1, kChunk); c += BLOCK)
+        all &= (flags[c] != 0) && (__ldg(&bodies[c * kChunk].w) == m0);
+    return __syncthreads_and(all) != 0;
+}
 
 // Output (A7: float4 stores) and split combine (A8), shared by every force-kernel variant: with
 // S > 1, each CTA writes its split partials, and the last CTA of a target tile (atomic ticket)
@@ -213,8 +318,8 @@ __device__ __forceinline__ void finish_targets(const ForceArgs& a, const IT& it,
     if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
 }
 
-template <int BLOCK, int R, bool kPacked, int CHUNK>
-__global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ ForceArgs a) {
+template <int BLOCK, int R, bool kPacked, int CHUNK, int MINB = 0, bool UNIT = false>
+__global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constant__ ForceArgs a) {
     __shared__ __align__(128) float4 sbuf[2][kTileJ];
     __shared__ __align__(8) uint64_t full[2];
     __shared__ int s_last;
@@ -222,6 +327,11 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
     const int tile = blockIdx.x;
     const int split = blockIdx.y;
     const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * R);
+
+    // ---- this split's source range [j0, j1)
+    const int64_t j0 = static_cast<int64_t>(split) * a.split_len;
+    const int64_t j1 = min(a.n_src, j0 + a.split_len);
+    const int ntiles = static_cast<int>(ceil_div<int64_t>(j1 - j0, kTileJ));
 
     // ---- this thread's targets (A3: one 128-bit read-only load each, coalesced)
     Interact<R, kPacked> it;
@@ -235,10 +345,14 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
     }
     it.zero_all();
 
-    // ---- this split's source range [j0, j1)
-    const int64_t j0 = static_cast<int64_t>(split) * a.split_len;
-    const int64_t j1 = min(a.n_src, j0 + a.split_len);
-    const int ntiles = static_cast<int>(ceil_div<int64_t>(j1 - j0, kTileJ));
+    // Mass-uniform splits run the UNIT instantiation, the others the per-body-mass one: the two
+    // are launched back to back over the same grid and each CTA leaves if its split is not its
+    // kind (the split combine below counts S arrivals per tile across both launches).
+    if (a.uniform != nullptr) {
+        if (split_mass_uniform<BLOCK>(a.bodies, a.uniform, j0, j1) != UNIT) return;
+    } else if (UNIT) {
+        return;
+    }
 
     if (threadIdx.x == 0) {
         mbar_init(&full[0], 1);
@@ -265,13 +379,23 @@ __global__ void __launch_bounds__(BLOCK) force_kernel(const __grid_constant__ Fo
         for (int c0 = 0; c0 < len; c0 += CHUNK) {
             const int c1 = min(len, c0 + CHUNK);
             it.chunk_begin();
-            if (c1 - c0 == CHUNK) {
+            if constexpr (UNIT) {
+                if (c1 - c0 == CHUNK) {
 #pragma unroll 4
-                for (int j = c0; j < c0 + CHUNK; ++j) it.body(sb[j], eps2);
+                    for (int j = c0; j < c0 + CHUNK; ++j) it.body_unit(sb[j], eps2);
+                } else {
+                    for (int j = c0; j < c1; ++j) it.body_unit(sb[j], eps2);
+                }
+                it.chunk_end_scaled(sb[c0].w);
             } else {
-                for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+                if (c1 - c0 == CHUNK) {
+#pragma unroll 4
+                    for (int j = c0; j < c0 + CHUNK; ++j) it.body(sb[j], eps2);
+                } else {
+                    for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+                }
+                it.chunk_end();
             }
-            it.chunk_end();
         }
         __syncthreads();                            // every lane is done reading this stage
         if (threadIdx.x == 0 && t + 2 < ntiles) issue(t + 2);
@@ -575,6 +699,8 @@ __global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_consta
     const int64_t j0 = static_cast<int64_t>(split) * a.split_len;
     const int64_t j1 = mn<int64_t>(a.n_src, j0 + a.split_len);
     const float eps2 = a.eps2;
+    // mass-uniform split: decided exactly as force_kernel decides it (same prepass flags)
+    const bool unit = a.uniform != nullptr && split_mass_uniform<BLOCK>(a.bodies, a.uniform, j0, j1);
     const float* bf = reinterpret_cast<const float*>(a.bodies);
     for (int64_t tb = j0; tb < j1; tb += kTileJ) {
         const int len = static_cast<int>(mn<int64_t>(kTileJ, j1 - tb));
@@ -602,6 +728,16 @@ __global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_consta
         for (int c0 = 0; c0 < len; c0 += a.chunk) {
             const int c1 = mn(len, c0 + a.chunk);
             it.chunk_begin();
+            if (unit) {
+                if (c1 - c0 == kChunk) {
+#pragma unroll 4
+                    for (int j = c0; j < c0 + kChunk; ++j) it.body_unit(src(j), eps2);
+                } else {
+                    for (int j = c0; j < c1; ++j) it.body_unit(src(j), eps2);
+                }
+                it.chunk_end_scaled(src(c0).w);
+                continue;
+            }
             if (c1 - c0 == kChunk) {
 #pragma unroll 4
                 for (int j = c0; j < c0 + kChunk; ++j) it.body(src(j), eps2);
@@ -645,8 +781,13 @@ static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
     const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
     dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
-    if (a.chunk == kChunk) force_kernel<BLOCK, R, kPacked, kChunk><<<grid, BLOCK, 0, stream>>>(a);
-    else force_kernel<BLOCK, R, kPacked, kChunkSmall><<<grid, BLOCK, 0, stream>>>(a);
+    if (a.chunk == kChunk) {
+        // mass-uniform splits, then the others (each CTA of either launch leaves unless its split is its kind)
+        if (a.uniform != nullptr) force_kernel<BLOCK, R, kPacked, kChunk, 0, true><<<grid, BLOCK, 0, stream>>>(a);
+        force_kernel<BLOCK, R, kPacked, kChunk><<<grid, BLOCK, 0, stream>>>(a);
+    } else {
+        force_kernel<BLOCK, R, kPacked, kChunkSmall><<<grid, BLOCK, 0, stream>>>(a);
+    }
     return cudaGetLastError();
 }
 
@@ -664,18 +805,29 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.chunk = chunk_len(n_src);
     a.split_len = chunks_per_split(n_src) * a.chunk;
     a.counters = static_cast<unsigned*>(ws);
-    a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count));
+    a.uniform = nullptr;
+    a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count) + flags_bytes(n_src));
 
     const LaunchOverride& ov = launch_override();
+    // n_src <= kSmallMaxSources: in-CTA splits (same arithmetic and order, see force_small_kernel);
+    // a block_threads / per_thread override selects the general kernel (used by the bit-identity test).
+    if (nbody_variant() == 0 && n_src <= kSmallMaxSources && ov.block_threads == 0 && ov.per_thread == 0)
+        return launch_small(a, stream);
+    if (a.splits > 1) {                               // tickets zeroed (+ mass-uniform chunk flags, R11)
+        uint8_t* flags = uses_chunk_flags(n_src) ? reinterpret_cast<uint8_t*>(static_cast<char*>(ws) + counters_bytes(tgt_count))
+                                                 : nullptr;
+        const int64_t ntiles = ceil_div<int64_t>(tgt_count, 128);
+        const int64_t work = flags ? ceil_div<int64_t>(ceil_div<int64_t>(n_src, kChunk), 8) : ceil_div<int64_t>(ntiles, 256);
+        const int grid = static_cast<int>(mx<int64_t>(1, mn<int64_t>(work, 4LL * device_num_sms())));
+        prepass_kernel<<<grid, 256, 0, stream>>>(bodies, n_src, flags, a.counters, ntiles);
+        a.uniform = flags;
+    }
     if (nbody_variant() != 0) {                       // F1 staging ablation (general mapping only)
         const int v = nbody_variant();
         if (ov.block_threads == 128 && ov.per_thread == 1) return launch_ablate<128, 1>(a, v, stream);
         if (ov.block_threads == 128) return launch_ablate<128, 2>(a, v, stream);
         return launch_ablate<256, 2>(a, v, stream);
     }
-    // n_src <= kSmallMaxSources: in-CTA splits (same arithmetic and order, see force_small_kernel);
-    // a block_threads / per_thread override selects the general kernel (used by the bit-identity test).
-    if (n_src <= kSmallMaxSources && ov.block_threads == 0 && ov.per_thread == 0) return launch_small(a, stream);
     int block = ov.block_threads, R = ov.per_thread;
     if (block == 0 || R == 0) {
         // Automatic (tools/tune_nbody.py sweep on B200, profiles/tune_nbody_r01.jsonl): 256 threads x

@@ -147,6 +147,12 @@ __global__ void __launch_bounds__(kBlock) force64_kernel(const __grid_constant__
         }
         ax[r] = sx; ay[r] = sy; az[r] = sz;
         store(a.accel + t, r);
+        // leave the workspace zero-filled (stale partials could sit where a later call keeps tickets)
+        for (int s = 0; s < a.splits; ++s) {
+            double2* q = reinterpret_cast<double2*>(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
+            __stcg(q, make_double2(0.0, 0.0));
+            __stcg(q + 1, make_double2(0.0, 0.0));
+        }
     }
     if (threadIdx.x == 0) a.counters[tile] = 0u;
 }

@@ -244,6 +244,9 @@ __global__ void __launch_bounds__(kBlock) bmap_kernel(const __grid_constant__ Ar
         Acc acc = const_cast<const Acc&>(vp[t]);
         for (int s = 1; s < a.splits; ++s) acc = acc_add(acc, const_cast<const Acc&>(vp[static_cast<int64_t>(s) * a.tgt_count + t]));
         a.out[t] = acc;
+        // leave the workspace zero-filled: stale partials could otherwise sit where a later call
+        // with other sizes keeps its tickets
+        for (int s = 0; s < a.splits; ++s) a.partial[static_cast<int64_t>(s) * a.tgt_count + t] = Acc{};
     }
     if (threadIdx.x == 0) a.counters[tile] = 0u;
 }

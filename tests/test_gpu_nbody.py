@@ -262,3 +262,63 @@ def test_momentum_after_ten_steps(lime):
         v = vel.cpu().numpy()[:, :3].astype(np.float64)
         P = (m[:, None] * v).sum(0)
         assert np.linalg.norm(P) <= 1e-6 * (m * np.linalg.norm(v, axis=1)).sum()
+
+
+# ------------------------------------------------- R11: mass-uniform splits (n_src > 8192)
+def _mixed_split_bodies(lime, n, seed, perturbed_splits):
+    """Equal masses 1/n (not a power of two) except in the listed splits, whose masses vary."""
+    b = inputs.nbody_bodies(n, seed=seed)
+    b[:, 3] = np.float32(1.0 / n)
+    S = lime.nbody_splits(n)
+    chunks = -(-n // 256)
+    split_len = -(-chunks // S) * 256                    # chunks_per_split * 256 (DESIGN.md R11)
+    rng = np.random.default_rng(seed)
+    for s in perturbed_splits:
+        lo, hi = s * split_len, min(n, (s + 1) * split_len)
+        b[lo:hi, 3] = (rng.uniform(0.5, 1.5, hi - lo) / n).astype(np.float32)
+    return b
+
+
+@pytest.mark.parametrize("n,perturbed", [(20000, []), (20000, [3, 7]), (50000, [0]), (50000, list(range(16)))])
+def test_mass_uniform_splits_match_oracle(lime, n, perturbed):
+    b = _mixed_split_bodies(lime, n, 300 + n, perturbed)
+    acc = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    rows = np.random.default_rng(n).choice(n, 300, replace=False)
+    rows = np.concatenate([rows, [0, n - 1]])
+    ref, mag = oracle.nbody_accel_rows(b, EPS2, rows, threads=8)
+    err = nbody_rel_err(acc[rows], ref, mag)
+    assert err.max() <= NBODY_RTOL, err.max()
+
+
+def test_mass_uniform_splits_bit_identity(lime):
+    # factored (mass-uniform) and per-body-mass splits in one call: shards, launch configurations
+    # and every staging-ablation variant must still agree bit for bit
+    n = 20000
+    b = _dev(_mixed_split_bodies(lime, n, 77, [2, 9, 15]))
+    full = lime.map_nbody(b, float(EPS2)).cpu()
+    for begin, count in [(0, 5000), (5000, 15000), (12345, 99)]:
+        assert torch.equal(lime.map_nbody(b, float(EPS2), begin, count).cpu(), full[begin:begin + count])
+    for block, R in [(128, 1), (128, 2), (256, 4), (256, 8)]:
+        with lime.launch_override(block_threads=block, per_thread=R):
+            assert torch.equal(lime.map_nbody(b, float(EPS2)).cpu(), full), (block, R)
+    for v in range(1, 6):
+        with lime.nbody_variant(v):
+            assert torch.equal(lime.map_nbody(b, float(EPS2)).cpu(), full), v
+
+
+def test_mass_uniform_edge_masses(lime):
+    # a massless body breaks its split's uniformity; an all-massless split contributes exactly 0
+    n = 1 << 14
+    rows = np.arange(0, n, 97)
+    b = inputs.nbody_bodies(n, seed=55)
+    b[n - 1, 3] = 0.0
+    acc = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    ref, mag = oracle.nbody_accel_rows(b, EPS2, rows, threads=8)
+    assert nbody_rel_err(acc[rows], ref, mag).max() <= NBODY_RTOL
+    S = lime.nbody_splits(n)
+    split_len = -(-(-(-n // 256)) // S) * 256
+    b[:split_len, 3] = 0.0                               # split 0 massless: uniform with m = 0
+    acc0 = lime.map_nbody(_dev(b), float(EPS2)).cpu().numpy()
+    ref0, mag0 = oracle.nbody_accel_rows(b, EPS2, rows, threads=8)
+    assert np.all(np.isfinite(acc0))
+    assert nbody_rel_err(acc0[rows], ref0, mag0).max() <= NBODY_RTOL
