@@ -29,9 +29,11 @@
  *   before returning (their outputs are host memory).
  * Workspaces. Entry points taking (ws, ws_bytes) need a device scratch buffer
  *   of at least the size returned by the matching *_workspace_bytes() query,
- *   ZERO-FILLED before its first use; every call leaves it zero-filled again
- *   (self-resetting counters), so one buffer can be reused by consecutive
- *   calls on the same stream. Two calls that run concurrently need two
+ *   ZERO-FILLED before its first use; every call leaves every word a later
+ *   call relies on zero again (self-resetting counters; split partials are
+ *   re-zeroed by the CTA that consumes them, and lime_map_nbody zeroes its own
+ *   tickets in a prepass), so one buffer can be reused by consecutive calls of
+ *   ANY sizes on the same stream. Two calls that run concurrently need two
  *   workspaces.
  * Errors. Every entry point returns lime_status; no C++ exception crosses the
  *   ABI. Validation order: arguments (LIME_ERR_INVALID_ARG) -> alignment
@@ -100,6 +102,13 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
  * else 256); each chunk is summed in j order into a chunk partial; chunk
  * partials are added in order into one of
  * S = nbody_splits(n_src) split partials; split partials are added in s order.
+ * Mass-uniform splits (n_src > 8192; R11): when every body of a
+ * split has the same mass m (bitwise-equal floats), each chunk partial is
+ * sum_j (p_j - p_i) / R^3 and is added as m * partial (exact algebra, one fewer
+ * FP32 multiply per interaction); for a power-of-two m this rounds exactly like
+ * the per-body form. A prepass kernel computes the per-chunk flags (and zeroes
+ * the split tickets) on `stream` before the force kernels.
+ * Range: the self term needs (eps2)^{-3/2} * max(m_j, 1) finite in fp32.
  * Launch override: grid ignored; block_threads in {128, 256}; per_thread in {1, 2, 4, 8}.
  * =========================================================================== */
 size_t lime_map_nbody_workspace_bytes(int64_t n_src, int64_t tgt_count);

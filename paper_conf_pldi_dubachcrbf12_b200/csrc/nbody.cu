@@ -464,7 +464,8 @@ __global__ void __launch_bounds__(32 * kMaxSplitsSmall) force_small_kernel(const
     __syncthreads();
     if (warp == 0 && valid) {
         float4 acc = part[lane];
-        for (int s = 1; s < a.splits; ++s) {
+#pragma unroll 8
+        for (int s = 1; s < a.splits; ++s) {       // unrolled: the LDS issue ahead of the in-order FADD chain
             const float4 p = part[s * 32 + lane];
             acc.x += p.x; acc.y += p.y; acc.z += p.z;
         }
@@ -557,6 +558,7 @@ __global__ void __launch_bounds__(32 * kMaxSplitsSmall) simulate_small_kernel(co
             __syncthreads();
             if (warp == 0 && valid) {
                 float4 acc = part[lane];
+#pragma unroll 8
                 for (int s = 1; s < a.splits; ++s) {
                     const float4 q = part[s * 32 + lane];
                     acc.x += q.x; acc.y += q.y; acc.z += q.z;
