@@ -406,17 +406,21 @@ __global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constan
 
 // =====================================================================================
 // Small problems (n_src <= kSmallMaxSources, e.g. the paper's 4096 bodies, Table 3): the
-// splits live inside one CTA instead of across CTAs. A CTA owns 32 targets (one per lane) and has
-// one warp per split; warp w bulk-copies split w's sources (<= 8 KB) into its own smem slice and
-// runs exactly the arithmetic of the general kernel (scalar variant: chunk partials added into
-// the split accumulator in chunk order); the split partials are then added in split order from
-// shared memory. Same summation order as force_kernel, hence bit-identical results, but no global
-// partials, no atomic tickets and ~16 warps per SM instead of 1-2 CTAs of 4 warps.
+// splits live inside one CTA instead of across CTAs. A CTA owns 32 targets; each warp owns TWO
+// consecutive splits, one per half-warp, and each lane of a half-warp carries a packed PAIR of the
+// CTA's targets (lane q of the half: targets 2q, 2q+1), so every FFMA2/FADD2/FMUL2 does two
+// interactions -- this launch is issue-bound, and packing halves the FP32 issue slots per
+// interaction. Warp w bulk-copies its two splits' sources (<= 2 x 4 KB, contiguous) into its smem
+// slice and runs exactly the arithmetic of the general kernel (chunk partials added into the split
+// accumulator in chunk order; each half of a packed op rounds exactly like the scalar op); the
+// split partials are then added in split order from shared memory. Same summation order as
+// force_kernel, hence bit-identical results, with no global partials and no atomic tickets.
 // =====================================================================================
-// One split's contribution for one target: chunk partials added into the split accumulator in chunk
-// order -- the arithmetic of force_kernel's scalar variant (shared by force_small_kernel and the
-// persistent simulation kernel, so all three agree bit for bit).
-__device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* sb, int len, int chunk, float eps2) {
+// One split's contribution for the lane's targets: chunk partials added into the split accumulator
+// in chunk order -- the arithmetic of force_kernel (shared by force_small_kernel and the persistent
+// simulation kernel, so all three agree bit for bit).
+template <class IT>
+__device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2) {
     for (int c0 = 0; c0 < len; c0 += chunk) {
         const int c1 = mn(len, c0 + chunk);
         it.chunk_begin();
@@ -433,36 +437,56 @@ __device__ __forceinline__ void split_sum(Interact<1, false>& it, const float4* 
     }
 }
 
-__global__ void __launch_bounds__(32 * kMaxSplitsSmall) force_small_kernel(const __grid_constant__ ForceArgs a) {
+// Lane -> (split, target pair) map of the small kernels: warp w, half h = lane / 16 works on split
+// 2w + h for the CTA's targets 2q and 2q + 1 (q = lane % 16).
+struct SmallLane {
+    int split, q;
+    __device__ __forceinline__ SmallLane() {
+        const unsigned lane = lane_id();
+        split = 2 * static_cast<int>(threadIdx.x >> 5) + static_cast<int>(lane >> 4);
+        q = static_cast<int>(lane & 15u);
+    }
+};
+
+__global__ void __launch_bounds__(16 * kMaxSplitsSmall) force_small_kernel(const __grid_constant__ ForceArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                          // [S][split_len]
     float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
-    __shared__ __align__(8) uint64_t bar[kMaxSplitsSmall];
+    __shared__ __align__(8) uint64_t bar[kMaxSplitsSmall / 2];
 
-    const int warp = threadIdx.x >> 5;            // = split index
+    const int warp = threadIdx.x >> 5;
     const unsigned lane = lane_id();
-    const int64_t t = static_cast<int64_t>(blockIdx.x) * 32 + lane;
-    const bool valid = t < a.tgt_count;
-    Interact<1, false> it;
-    it.set(0, __ldg(a.bodies + a.tgt_begin + (valid ? t : a.tgt_count - 1)));
+    const SmallLane sl;
+    const int64_t tg = static_cast<int64_t>(blockIdx.x) * 32;
+    Interact<2, true> it;
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+        const int64_t t = tg + 2 * sl.q + r;
+        it.set(r, __ldg(a.bodies + a.tgt_begin + (t < a.tgt_count ? t : a.tgt_count - 1)));
+    }
     it.zero_all();
 
-    const int64_t j0 = static_cast<int64_t>(warp) * a.split_len;
-    const int64_t j1 = mn<int64_t>(a.n_src, j0 + a.split_len);
-    const int len = static_cast<int>(j1 - j0);
-    float4* sb = src + static_cast<int64_t>(warp) * a.split_len;
+    // this warp's two splits: one contiguous source range
+    const int64_t w0 = static_cast<int64_t>(2 * warp) * a.split_len;
+    const int64_t w1 = mn<int64_t>(a.n_src, w0 + 2 * a.split_len);
     if (lane == 0) {
         mbar_init(&bar[warp], 1);
         fence_mbar_init();
-        mbar_arrive_expect_tx(&bar[warp], static_cast<uint32_t>(len) * 16u);
-        bulk_g2s(sb, a.bodies + j0, static_cast<uint32_t>(len) * 16u, &bar[warp]);
+        mbar_arrive_expect_tx(&bar[warp], static_cast<uint32_t>(w1 - w0) * 16u);
+        bulk_g2s(src + w0, a.bodies + w0, static_cast<uint32_t>(w1 - w0) * 16u, &bar[warp]);
     }
     __syncwarp();
     mbar_wait(&bar[warp], 0);
-    split_sum(it, sb, len, a.chunk, a.eps2);
-    part[warp * 32 + lane] = it.result(0);
+    const int64_t j0 = static_cast<int64_t>(sl.split) * a.split_len;
+    const int len = sl.split < a.splits ? static_cast<int>(mn<int64_t>(a.n_src, j0 + a.split_len) - j0) : 0;
+    split_sum(it, src + j0, len, a.chunk, a.eps2);
+    if (sl.split < a.splits) {
+        part[sl.split * 32 + 2 * sl.q] = it.result(0);
+        part[sl.split * 32 + 2 * sl.q + 1] = it.result(1);
+    }
     __syncthreads();
-    if (warp == 0 && valid) {
+    const int64_t t = tg + lane;
+    if (warp == 0 && t < a.tgt_count) {
         float4 acc = part[lane];
 #pragma unroll 8
         for (int s = 1; s < a.splits; ++s) {       // unrolled: the LDS issue ahead of the in-order FADD chain
@@ -484,7 +508,7 @@ static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
         attr = kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16;
     }
     const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
-    force_small_kernel<<<static_cast<unsigned>(ctas), 32 * a.splits, smem, stream>>>(a);
+    force_small_kernel<<<static_cast<unsigned>(ctas), 32 * ceil_div(a.splits, 2), smem, stream>>>(a);
     return cudaGetLastError();
 }
 
@@ -529,32 +553,41 @@ __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(32 * kMaxSplitsSmall) simulate_small_kernel(const __grid_constant__ SimArgs a) {
+__global__ void __launch_bounds__(16 * kMaxSplitsSmall) simulate_small_kernel(const __grid_constant__ SimArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                                   // [S][split_len]
     float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
-    const int warp = threadIdx.x >> 5;                // = split index
+    const int warp = threadIdx.x >> 5;                // owns splits 2 warp, 2 warp + 1 (force_small_kernel's map)
     const unsigned lane = lane_id();
+    const SmallLane sl;
     const int64_t groups = ceil_div<int64_t>(a.n, 32);
-    const int64_t j0 = static_cast<int64_t>(warp) * a.split_len;
-    const int len = static_cast<int>(mn<int64_t>(a.n, j0 + a.split_len) - j0);
-    float4* sb = src + j0;
+    const int64_t w0 = static_cast<int64_t>(2 * warp) * a.split_len;
+    const int wlen = static_cast<int>(mn<int64_t>(a.n, w0 + 2 * a.split_len) - w0);
+    const int64_t j0 = static_cast<int64_t>(sl.split) * a.split_len;
+    const int len = sl.split < a.splits ? static_cast<int>(mn<int64_t>(a.n, j0 + a.split_len) - j0) : 0;
     unsigned barrier_target = 0;
 
     for (int32_t k = 0; k < a.steps; ++k) {
         const float4* cur = (k & 1) ? a.pos_alt : a.pos;
         float4* nxt = (k & 1) ? a.pos : a.pos_alt;
-        for (int j = static_cast<int>(lane); j < len; j += 32) sb[j] = __ldcg(cur + j0 + j);
+        for (int j = static_cast<int>(lane); j < wlen; j += 32) src[w0 + j] = __ldcg(cur + w0 + j);
         __syncwarp();
         for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
             const int64_t t = g * 32 + lane;
             const bool valid = t < a.n;
             const float4 p = __ldcg(cur + (valid ? t : a.n - 1));
-            Interact<1, false> it;
-            it.set(0, p);
+            Interact<2, true> it;
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int64_t tr = g * 32 + 2 * sl.q + r;
+                it.set(r, __ldcg(cur + (tr < a.n ? tr : a.n - 1)));
+            }
             it.zero_all();
-            split_sum(it, sb, len, a.chunk, a.eps2);
-            part[warp * 32 + lane] = it.result(0);
+            split_sum(it, src + j0, len, a.chunk, a.eps2);
+            if (sl.split < a.splits) {
+                part[sl.split * 32 + 2 * sl.q] = it.result(0);
+                part[sl.split * 32 + 2 * sl.q + 1] = it.result(1);
+            }
             __syncthreads();
             if (warp == 0 && valid) {
                 float4 acc = part[lane];
@@ -629,7 +662,7 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.split_len = chunks_per_split(n) * a.chunk;
     a.eps2 = eps2;
     a.dt = dt;
-    const int block = 32 * a.splits;
+    const int block = 32 * ceil_div(a.splits, 2);
     const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
     static bool attr = false;
     if (!attr) {
