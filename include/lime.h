@@ -109,7 +109,8 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
  * the per-body form. A prepass kernel computes the per-chunk flags (and zeroes
  * the split tickets) on `stream` before the force kernels.
  * Range: the self term needs (eps2)^{-3/2} * max(m_j, 1) finite in fp32.
- * Launch override: grid ignored; block_threads in {128, 256}; per_thread in {1, 2, 4, 8}.
+ * Launch override: grid ignored; block_threads in {128, 256} with per_thread in {1, 2, 4, 8},
+ * or block_threads 512 with per_thread in {2, 4}.
  * =========================================================================== */
 size_t lime_map_nbody_workspace_bytes(int64_t n_src, int64_t tgt_count);
 /* Staging ablation (the paper's Fig. 8 memory-mapping variants, L391-398,

@@ -811,17 +811,20 @@ static cudaError_t launch_ablate(const ForceArgs& a, int v, cudaStream_t stream)
     return cudaGetLastError();
 }
 
+// MINB: 512-thread CTAs get __launch_bounds__(512, 1) (up to 128 registers: R = 4 compiles to 112,
+// one CTA = 16 warps per SM); the others leave the register choice to ptxas.
 template <int BLOCK, int R>
 static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
+    constexpr int MINB = BLOCK == 512 ? 1 : 0;
     const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
     dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
     if (a.chunk == kChunk) {
         // mass-uniform splits, then the others (each CTA of either launch leaves unless its split is its kind)
-        if (a.uniform != nullptr) force_kernel<BLOCK, R, kPacked, kChunk, 0, true><<<grid, BLOCK, 0, stream>>>(a);
-        force_kernel<BLOCK, R, kPacked, kChunk><<<grid, BLOCK, 0, stream>>>(a);
+        if (a.uniform != nullptr) force_kernel<BLOCK, R, kPacked, kChunk, MINB, true><<<grid, BLOCK, 0, stream>>>(a);
+        force_kernel<BLOCK, R, kPacked, kChunk, MINB><<<grid, BLOCK, 0, stream>>>(a);
     } else {
-        force_kernel<BLOCK, R, kPacked, kChunkSmall><<<grid, BLOCK, 0, stream>>>(a);
+        force_kernel<BLOCK, R, kPacked, kChunkSmall, MINB><<<grid, BLOCK, 0, stream>>>(a);
     }
     return cudaGetLastError();
 }
@@ -865,18 +868,27 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     }
     int block = ov.block_threads, R = ov.per_thread;
     if (block == 0 || R == 0) {
-        // Automatic (tools/tune_nbody.py sweep on B200, profiles/tune_nbody_r01.jsonl): 256 threads x
-        // 2 targets (one packed pair) is fastest at 2^20; small problems drop to 128-thread tiles so
-        // that there are >= 1.5 work items per SM.
+        // Automatic (B200 sweeps: tools/tune_nbody.py, tools/nbody_occ.cu; profiles/tune_nbody_r01.jsonl,
+        // profiles/experiments/nbody_unit_sweep_r01*.jsonl): 512 threads x 4 targets (two packed pairs,
+        // 112 registers, one CTA per SM) is fastest at 2^17..2^20 targets -- 47.6 vs 49.5 ms for
+        // 256 x 2 on the config-5 shard -- and is taken when it still fills >= 6 waves; otherwise
+        // 256 x 2, then 128-thread tiles so that there are >= 1.5 work items per SM.
         const int64_t want = 3LL * device_num_sms() / 2;
-        const int cand[][2] = {{256, 2}, {128, 2}, {128, 1}};
-        int pick = 2;
-        for (int k = 0; k < 3; ++k) {
+        const int cand[][2] = {{512, 4}, {256, 2}, {128, 2}, {128, 1}};
+        const int64_t need[] = {6LL * device_num_sms(), want, want, 0};
+        int pick = 3;
+        for (int k = 0; k < 4; ++k) {
             const int64_t items = ceil_div<int64_t>(tgt_count, cand[k][0] * cand[k][1]) * a.splits;
-            if (items >= want) { pick = k; break; }
+            if (items >= need[k]) { pick = k; break; }
         }
         if (block == 0) block = cand[pick][0];
         if (R == 0) R = cand[pick][1];
+    }
+    if (block == 512) {
+        switch (R) {
+            case 2: return launch_one<512, 2>(a, stream);
+            case 4: return launch_one<512, 4>(a, stream);
+        }
     }
     if (block == 256) {
         switch (R) {

@@ -37,11 +37,10 @@ def test_shards_are_slices_and_launch_independent(lime):
     for begin, count in [(0, 1), (1, 1000), (2048, 2049), (4000, 97), (17, 0)]:
         part = lime.map_nbody(b, float(EPS2), begin, count).cpu()
         assert torch.equal(part, full[begin:begin + count])
-    for block in (128, 256):
-        for R in (1, 2, 4, 8):
-            with lime.launch_override(block_threads=block, per_thread=R):
-                alt = lime.map_nbody(b, float(EPS2)).cpu()
-            assert torch.equal(alt, full), (block, R)
+    for block, R in [(b_, r_) for b_ in (128, 256) for r_ in (1, 2, 4, 8)] + [(512, 2), (512, 4)]:
+        with lime.launch_override(block_threads=block, per_thread=R):
+            alt = lime.map_nbody(b, float(EPS2)).cpu()
+        assert torch.equal(alt, full), (block, R)
 
 
 def test_p_way_sharding_bit_identical(lime):
@@ -298,7 +297,7 @@ def test_mass_uniform_splits_bit_identity(lime):
     full = lime.map_nbody(b, float(EPS2)).cpu()
     for begin, count in [(0, 5000), (5000, 15000), (12345, 99)]:
         assert torch.equal(lime.map_nbody(b, float(EPS2), begin, count).cpu(), full[begin:begin + count])
-    for block, R in [(128, 1), (128, 2), (256, 4), (256, 8)]:
+    for block, R in [(128, 1), (128, 2), (256, 2), (256, 4), (256, 8), (512, 2), (512, 4)]:
         with lime.launch_override(block_threads=block, per_thread=R):
             assert torch.equal(lime.map_nbody(b, float(EPS2)).cpu(), full), (block, R)
     for v in range(1, 6):

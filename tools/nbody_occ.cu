@@ -105,7 +105,21 @@ int main(int argc, char** argv) {
         fflush(stdout);
     }
     run(force_kernel<256, 2, true, kChunk, 0, false>, 256, 2, 0);    // per-body-mass instantiation alone
-    if (argc > 3) {
+    if (argc > 3 && argv[3][0] == 'u') {              // mass-uniform instantiations (equal masses)
+        run(force_kernel<256, 2, true, kChunk, 0, true>, 256, 2, 0);
+        run(force_kernel<256, 4, true, kChunk, 3, true>, 256, 4, 3);
+        run(force_kernel<256, 4, true, kChunk, 2, true>, 256, 4, 2);
+        run(force_kernel<128, 4, true, kChunk, 5, true>, 128, 4, 5);
+        run(force_kernel<128, 4, true, kChunk, 4, true>, 128, 4, 4);
+        run(force_kernel<128, 8, true, kChunk, 3, true>, 128, 8, 3);
+        run(force_kernel<256, 8, true, kChunk, 1, true>, 256, 8, 1);
+        run(force_kernel<512, 2, true, kChunk, 2, true>, 512, 2, 2);
+        run(force_kernel<512, 2, true, kChunk, 1, true>, 512, 2, 1);
+        run(force_kernel<512, 4, true, kChunk, 1, true>, 512, 4, 1);
+        run(force_kernel<64, 4, true, kChunk, 6, true>, 64, 4, 6);
+        run(force_kernel<64, 4, true, kChunk, 8, true>, 64, 4, 8);
+        run(force_kernel<256, 4, true, kChunk, 3, false>, 256, 4, 3);    // (per-body mass form, for the record)
+    } else if (argc > 3) {
         run(force_kernel<256, 2, true, kChunk, 1>, 256, 2, 1);
         run(force_kernel<256, 2, true, kChunk, 4>, 256, 2, 4);
         run(force_kernel<256, 2, true, kChunk, 5>, 256, 2, 5);
