@@ -24,8 +24,8 @@ namespace parboil {
 constexpr int kChunk = 256;
 constexpr int kMaxSplits = 16;
 constexpr int kTileJ = 1024;     // sources per smem stage (16 KB)
-constexpr int kBlock = 128;
-constexpr int kU = 4;            // targets per thread (two packed pairs)
+constexpr int kBlock = 64;       // smallest target-tile block (workspace ticket sizing)
+constexpr int kUMin = 2;         // fewest targets per thread of any element type (ticket sizing)
 
 int64_t chunks_per_split(int64_t n_src) {
     const int64_t chunks = ceil_div<int64_t>(n_src, kChunk);
@@ -37,13 +37,21 @@ int splits(int64_t n_src) {
     return static_cast<int>(ceil_div<int64_t>(chunks, chunks_per_split(n_src)));
 }
 static size_t counters_bytes(int64_t targets) {
-    return ((ceil_div<int64_t>(targets, kBlock * kU) * 4 + 255) / 256) * 256;
+    return ((ceil_div<int64_t>(targets, kBlock * kUMin) * 4 + 255) / 256) * 256;
 }
 
 // ------------------------------------------------------------------ element policies
 // CP: targets are lattice points t -> (ix, iy) = (t % nx, t / nx); one fp32 accumulator each.
+#ifndef CP_BLOCK
+#define CP_BLOCK 128
+#endif
+#ifndef CP_U
+#define CP_U 4
+#endif
 struct CP {
     using Acc = float;
+    static constexpr int kBlock = CP_BLOCK;
+    static constexpr int kU = CP_U;  // targets per thread (packed pairs)
     struct Params {
         int32_t nx;
         float z, h;
@@ -92,8 +100,20 @@ struct CP {
 };
 
 // MRI-Q: targets are voxels [X][3]; sources are (kx, ky, kz, phiMag) prepared by phimag_kernel.
+// MRI-Q tile: 128 threads x 2 targets (one packed pair per thread) -- B200 sweep (tools/tune_parboil.py
+// over -DMRIQ_BLOCK / -DMRIQ_U A/B builds, profiles/experiments/tune_parboil_r01.txt): 66.7 us vs 72.7 us
+// for 128 x 4; twice the warps of the 4-target tile hide the MUFU.SIN/COS latency better. Results do
+// not depend on it (the summation order follows the source chunking only).
+#ifndef MRIQ_BLOCK
+#define MRIQ_BLOCK 128
+#endif
+#ifndef MRIQ_U
+#define MRIQ_U 2
+#endif
 struct MRIQ {
     using Acc = float2;
+    static constexpr int kBlock = MRIQ_BLOCK;
+    static constexpr int kU = MRIQ_U;
     struct Params {
         const float* voxels;
     };
@@ -158,8 +178,8 @@ struct Args {
 __device__ __forceinline__ float acc_add(float a, float b) { return a + b; }
 __device__ __forceinline__ float2 acc_add(float2 a, float2 b) { return make_float2(a.x + b.x, a.y + b.y); }
 
-template <class E>
-__global__ void __launch_bounds__(kBlock) bmap_kernel(const __grid_constant__ Args<E> a) {
+template <class E, int BLOCK>
+__global__ void __launch_bounds__(BLOCK) bmap_kernel(const __grid_constant__ Args<E> a) {
     __shared__ __align__(128) float4 sbuf[2][kTileJ];
     __shared__ __align__(8) uint64_t full[2];
     __shared__ int s_last;
@@ -167,12 +187,12 @@ __global__ void __launch_bounds__(kBlock) bmap_kernel(const __grid_constant__ Ar
 
     const int tile = blockIdx.x;
     const int split = blockIdx.y;
-    const int64_t tbase = static_cast<int64_t>(tile) * (kBlock * kU);
+    const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * E::kU);
     typename E::Tgt tg;
-    bool valid[kU];
+    bool valid[E::kU];
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * kBlock;
+    for (int u = 0; u < E::kU; ++u) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * BLOCK;
         valid[u] = t < a.tgt_count;
         E::make_target(a.p, nullptr, a.tgt_begin + (valid[u] ? t : a.tgt_count - 1), u, tg);
     }
@@ -219,15 +239,15 @@ __global__ void __launch_bounds__(kBlock) bmap_kernel(const __grid_constant__ Ar
 
     if (a.splits == 1) {
 #pragma unroll
-        for (int u = 0; u < kU; ++u) {
-            const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * kBlock;
+        for (int u = 0; u < E::kU; ++u) {
+            const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * BLOCK;
             if (valid[u]) a.out[t] = E::get(st, u);
         }
         return;
     }
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * kBlock;
+    for (int u = 0; u < E::kU; ++u) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * BLOCK;
         if (valid[u]) a.partial[static_cast<int64_t>(split) * a.tgt_count + t] = E::get(st, u);
     }
     __threadfence();
@@ -237,8 +257,8 @@ __global__ void __launch_bounds__(kBlock) bmap_kernel(const __grid_constant__ Ar
     if (!s_last) return;
     __threadfence();
 #pragma unroll
-    for (int u = 0; u < kU; ++u) {
-        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * kBlock;
+    for (int u = 0; u < E::kU; ++u) {
+        const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(u) * BLOCK;
         if (!valid[u]) continue;
         const volatile Acc* vp = a.partial;
         Acc acc = const_cast<const Acc&>(vp[t]);
@@ -266,9 +286,15 @@ static cudaError_t launch_bmap(Args<E>& a, void* ws, cudaStream_t stream) {
     a.split_len = chunks_per_split(a.n_src) * kChunk;
     a.counters = static_cast<unsigned*>(ws);
     a.partial = reinterpret_cast<typename E::Acc*>(static_cast<char*>(ws) + counters_bytes(a.tgt_count));
-    const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(kBlock) * kU);
+    // target-tile width: E::kBlock threads x kU targets by default (tools/tune_parboil.py sweep);
+    // a block_threads override of 64 / 128 / 256 selects another (results never depend on it)
+    int block = launch_override().block_threads;
+    if (block != 64 && block != 128 && block != 256) block = E::kBlock;
+    const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(block) * E::kU);
     dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
-    bmap_kernel<E><<<grid, kBlock, 0, stream>>>(a);
+    if (block == 64) bmap_kernel<E, 64><<<grid, 64, 0, stream>>>(a);
+    else if (block == 128) bmap_kernel<E, 128><<<grid, 128, 0, stream>>>(a);
+    else bmap_kernel<E, 256><<<grid, 256, 0, stream>>>(a);
     return cudaGetLastError();
 }
 
