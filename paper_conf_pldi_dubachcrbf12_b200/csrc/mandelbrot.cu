@@ -39,6 +39,14 @@ struct Args {
 // ptxas contracts packed mul.rn/add.rn.f32x2 pairs into FFMA2 even with --fmad=false (observed
 // on CUDA 12.9, see tests/test_sass_guards.py), which changes rounding; an FFMA2 cannot be
 // contracted further, so this spelling keeps one IEEE rounding per operation of R7.
+// n += alive as ONE predicated integer add per pixel: the sticky FSETP.LE.AND's predicate guards
+// the add directly (the C++ spellings `n += a`, `if (a) n++` compile to two IADD3 per pixel on
+// CUDA 12.9, and this loop is issue-bound: 8 packed FP32 ops = 16 pipe cycles per iteration
+// against ~15 issued instructions).
+__device__ __forceinline__ void count(int& n, bool alive) {
+    asm("{ .reg .pred p; setp.ne.b16 p, %1, 0; @p add.s32 %0, %0, 1; }" : "+r"(n) : "h"(static_cast<short>(alive)));
+}
+
 struct State {
     float2 x, y, cx, cy;
     int n0, n1;
@@ -50,8 +58,8 @@ struct State {
         const float2 s = fma2(xx, one, yy);          // x^2 + y^2
         a0 = a0 && (s.x <= 4.0f);                    // test before the update (R7); sticky once escaped
         a1 = a1 && (s.y <= 4.0f);
-        n0 += a0 ? 1 : 0;
-        n1 += a1 ? 1 : 0;
+        count(n0, a0);
+        count(n1, a1);
         const float2 xy = fma2(x, y, z);
         x = fma2(fma2(yy, mone, xx), one, cx);       // x <- (x^2 - y^2) + cx
         y = fma2(fma2(xy, one, xy), one, cy);        // y <- (xy + xy) + cy
