@@ -193,7 +193,8 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
     __threadfence();
     if (warp == 0) {
         double bx = 0.0, by = 0.0;
-        for (unsigned k = lane_id(); k < gridDim.x; k += 32) {
+#pragma unroll 8
+        for (unsigned k = lane_id(); k < gridDim.x; k += 32) {   // unrolled: the L2 loads issue ahead of the adds
             const double2 p = __ldcg(partial + k);
             bx += p.x;
             by += p.y;

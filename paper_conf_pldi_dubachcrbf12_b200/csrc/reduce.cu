@@ -160,7 +160,8 @@ __global__ void __launch_bounds__(256) reduce_kernel(const T* __restrict__ x, in
         // fixed order (deterministic for a given grid): lane l folds partials l, l+32, ... in index
         // order, then the fixed xor-shuffle tree combines the 32 lane values
         A b = P::id();
-        for (unsigned k = lane_id(); k < gridDim.x; k += 32) b = P::comb(b, ldcg_acc(partial + k));
+#pragma unroll 8
+        for (unsigned k = lane_id(); k < gridDim.x; k += 32) b = P::comb(b, ldcg_acc(partial + k));   // loads issue ahead
         b = warp_reduce<P>(b);
         if (lane_id() == 0) {
             if constexpr (OP != kSum && std::is_floating_point<T>::value) {

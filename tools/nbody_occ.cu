@@ -105,7 +105,16 @@ int main(int argc, char** argv) {
         fflush(stdout);
     }
     run(force_kernel<256, 2, true, kChunk, 0, false>, 256, 2, 0);    // per-body-mass instantiation alone
-    if (argc > 3 && argv[3][0] == 'u') {              // mass-uniform instantiations (equal masses)
+    if (argc > 3 && argv[3][0] == 'w') {              // wide tiles (mass-uniform, equal masses)
+        run(force_kernel<512, 4, true, kChunk, 1, true>, 512, 4, 1);
+        run(force_kernel<384, 4, true, kChunk, 1, true>, 384, 4, 1);
+        run(force_kernel<384, 6, true, kChunk, 1, true>, 384, 6, 1);
+        run(force_kernel<256, 6, true, kChunk, 1, true>, 256, 6, 1);
+        run(force_kernel<256, 6, true, kChunk, 2, true>, 256, 6, 2);
+        run(force_kernel<320, 4, true, kChunk, 1, true>, 320, 4, 1);
+        run(force_kernel<448, 4, true, kChunk, 1, true>, 448, 4, 1);
+        run(force_kernel<512, 4, true, kChunk, 1, false>, 512, 4, 1);   // per-body-mass form
+    } else if (argc > 3 && argv[3][0] == 'u') {       // mass-uniform instantiations (equal masses)
         run(force_kernel<256, 2, true, kChunk, 0, true>, 256, 2, 0);
         run(force_kernel<256, 4, true, kChunk, 3, true>, 256, 4, 3);
         run(force_kernel<256, 4, true, kChunk, 2, true>, 256, 4, 2);
