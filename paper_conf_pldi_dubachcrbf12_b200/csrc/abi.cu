@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "../../include/lime.h"
@@ -20,6 +21,10 @@ static thread_local int g_nbody_variant = 0;
 
 const LaunchOverride& launch_override() { return g_override; }
 int nbody_variant() { return g_nbody_variant; }
+bool pdl_enabled() {
+    static const bool on = std::getenv("LIME_NO_PDL") == nullptr;
+    return on;
+}
 
 int device_num_sms() {
     static int cached[64] = {0};

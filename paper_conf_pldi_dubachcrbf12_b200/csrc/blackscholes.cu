@@ -3,16 +3,20 @@
 // BASELINE.json config 2 (not in the paper; R5-R6). A3/A7: 128-bit read-only
 // streaming loads of the SoA operands (ld.global.nc.L1::no_allocate, PAPER.md L267-275
 // vectorisation of read-only arrays) and evict-first 128-bit stores. A8: the fused
-// variant never writes call/put; fp64 partials per thread -> warp shuffle -> CTA ->
-// last CTA combines CTA partials in index order.
+// variant never writes call/put; fp32 partials per thread -> fp64 from the warp up -> CTA ->
+// last CTA combines CTA partials in index order. Both kernels are launched with programmatic
+// dependent launch (common.cuh pdl_enter/launch_pdl), so back-to-back launches overlap the
+// next grid's launch with this one's drain.
 //
-// The element function is written for B200's ridge point: 6 MUFU and ~48
-// FP32 lane-ops per option, two options per packed FFMA2/FMUL2 instruction. Savings vs the
-// textbook evaluation:
+// The element function is written for B200's ridge point: 6 MUFU per option,
+// two options per packed FFMA2/FMUL2 instruction. Savings vs the textbook evaluation:
 //   * 1/(sigma sqrt T) = rsqrt(T) / sigma  (one MUFU.RSQ gives both sqrt T and its inverse)
 //   * ln(S/X) = (lg2 S - lg2 X) ln 2
 //   * K phi(d2) = S phi(d1) (exact identity, K = X e^{-rT}) -> one exponential serves both
 //     normal-CDF tails (Abramowitz & Stegun 26.2.17, |err| < 7.5e-8).
+// The map evaluates call and put per option (price2, ~48 FP32 lane-ops); the fused sums use
+// price2_wu (~34 lane-ops, no per-option selects), which sums w and u with call = w + u/2 and
+// put = w - u/2.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -24,6 +28,10 @@ struct Consts {
     float inv_sigma;        // 1/sigma
     float sigma;
     float neg_r_log2e;      // -r log2(e)
+    // fused map+reduce element (price2_wu): ln 2 folded into the d1/d2 constants
+    float a_l2;             // (r + sigma^2/2) / ln 2
+    float b_l2;             // (r - sigma^2/2) / ln 2
+    float ln2_over_sigma;   // ln 2 / sigma
 };
 
 constexpr float kLn2 = 0.693147180559945309f;
@@ -88,6 +96,48 @@ __device__ __forceinline__ P2 price2(float2 S, float2 X, float2 T, const Consts&
     return r;
 }
 
+// ---- fused map+reduce element: the two sums need no per-option call/put selects.
+// With A = S N(d1) - S/2 = copysign(S/2 - S N(-|d1|), d1) and B = K N(d2) - K/2 (same form),
+//   call = w + u/2, put = w - u/2,  where w = A - B, u = S - K
+// (put = call - S + K, put-call parity, holds by construction). The kernel sums w and u only.
+// Per option: 6 MUFU as in price2, ~34 FP32 lane-ops (ln 2 and 1/sqrt(2 pi) folded into the
+// constants; the AS polynomial carries the sign so S/2 - S N(-|d1|) is one FFMA), 2 LOP3.
+constexpr float kASn_a1 = -kAS_a1 * kInvSqrt2Pi;
+constexpr float kASn_a2 = -kAS_a2 * kInvSqrt2Pi;
+constexpr float kASn_a3 = -kAS_a3 * kInvSqrt2Pi;
+constexpr float kASn_a4 = -kAS_a4 * kInvSqrt2Pi;
+constexpr float kASn_a5 = -kAS_a5 * kInvSqrt2Pi;
+__device__ __forceinline__ float2 as_poly2n(float2 k) {   // -phi-scaled AS polynomial: -poly(k)/sqrt(2 pi)
+    float2 p = fma2(k, bcast2(kASn_a5), bcast2(kASn_a4));
+    p = fma2(k, p, bcast2(kASn_a3));
+    p = fma2(k, p, bcast2(kASn_a2));
+    p = fma2(k, p, bcast2(kASn_a1));
+    return mul2(k, p);
+}
+__device__ __forceinline__ void price2_wu(float2 S, float2 X, float2 T, const Consts& c, float2& w, float2& u) {
+    const float2 rsT = make_float2(rsqrt_approx(T.x), rsqrt_approx(T.y));
+    const float2 q = mul2(rsT, bcast2(c.ln2_over_sigma));                // ln 2 / (sigma sqrt T)
+    const float2 lg = sub2(make_float2(lg2_approx(S.x), lg2_approx(S.y)),
+                           make_float2(lg2_approx(X.x), lg2_approx(X.y)));  // log2(S/X)
+    const float2 d1 = mul2(fma2(bcast2(c.a_l2), T, lg), q);
+    const float2 d2 = mul2(fma2(bcast2(c.b_l2), T, lg), q);
+    const float2 er = mul2(bcast2(c.neg_r_log2e), T);
+    const float2 K = mul2(X, make_float2(ex2_approx(er.x), ex2_approx(er.y)));   // X e^{-rT}
+    const float2 D1 = fma2(bcast2(kAS_p), abs2(d1), bcast2(1.f));
+    const float2 D2 = fma2(bcast2(kAS_p), abs2(d2), bcast2(1.f));
+    const float2 DD = mul2(D1, D2);
+    const float2 rr = make_float2(rcp_approx(DD.x), rcp_approx(DD.y));
+    const float2 k1 = mul2(D2, rr);                                     // 1 / D1
+    const float2 k2 = mul2(D1, rr);                                     // 1 / D2
+    const float2 g = mul2(mul2(bcast2(kNegHalfLog2e), d1), d1);
+    const float2 se = mul2(S, make_float2(ex2_approx(g.x), ex2_approx(g.y)));   // S phi(d1) sqrt(2 pi)
+    const float2 a = fma2(bcast2(0.5f), S, mul2(se, as_poly2n(k1)));   // S/2 - S N(-|d1|)
+    const float2 b = fma2(bcast2(0.5f), K, mul2(se, as_poly2n(k2)));   // K/2 - K N(-|d2|)
+    w = sub2(make_float2(copysignf(a.x, d1.x), copysignf(a.y, d1.y)),
+             make_float2(copysignf(b.x, d2.x), copysignf(b.y, d2.y)));
+    u = sub2(S, K);
+}
+
 __device__ __forceinline__ void price(float S, float X, float T, const Consts& c, float& call, float& put) {
     const P2 r = price2(bcast2(S), bcast2(X), bcast2(T), c);
     call = r.call.x;
@@ -102,28 +152,39 @@ __device__ __forceinline__ void price4(const float4& s, const float4& x, const f
     pv = make_float4(a.put.x, a.put.y, b.put.x, b.put.y);
 }
 
-__global__ void __launch_bounds__(256, 4) map_kernel(const float* __restrict__ S, const float* __restrict__ X,
-                                                  const float* __restrict__ T, int64_t n, Consts c,
-                                                  float* __restrict__ call, float* __restrict__ put) {
-    const int64_t n4 = n >> 2;
-    const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
-    const float4* S4 = reinterpret_cast<const float4*>(S);
-    const float4* X4 = reinterpret_cast<const float4*>(X);
-    const float4* T4 = reinterpret_cast<const float4*>(T);
-    int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
+// Grid-stride sweep over the float4 groups [i, n4), software-pipelined one iteration ahead: the
+// next group's 48 B are loaded before this one is priced. (A copy-free two-buffer ring measured
+// 1-2 us slower for the fused kernel and 3-5 us for the map: ptxas sinks the ring's look-ahead loads
+// below the pricing at the 64-register cap, tools/bs_pdl.cu, profiles/experiments/bs_pdl_loop_r01m.jsonl.)
+template <typename F>
+__device__ __forceinline__ void sweep_groups(const float4* __restrict__ S4, const float4* __restrict__ X4,
+                                             const float4* __restrict__ T4, int64_t i, int64_t n4, int64_t stride,
+                                             F&& body) {
     float4 s, x, t;
     if (i < n4) { s = ld_stream_f4(S4 + i); x = ld_stream_f4(X4 + i); t = ld_stream_f4(T4 + i); }
     for (; i < n4; i += stride) {
-        // software pipeline: issue the next iteration's 48 B of loads before pricing this one
         const int64_t nx = i + stride;
         float4 s2 = s, x2 = x, t2 = t;
         if (nx < n4) { s2 = ld_stream_f4(S4 + nx); x2 = ld_stream_f4(X4 + nx); t2 = ld_stream_f4(T4 + nx); }
-        float4 cv, pv;
-        price4(s, x, t, c, cv, pv);
-        st_stream_f4(reinterpret_cast<float4*>(call) + i, cv);
-        st_stream_f4(reinterpret_cast<float4*>(put) + i, pv);
+        body(i, s, x, t);
         s = s2; x = x2; t = t2;
     }
+}
+
+__global__ void __launch_bounds__(256, 4) map_kernel(const float* __restrict__ S, const float* __restrict__ X,
+                                                  const float* __restrict__ T, int64_t n, Consts c,
+                                                  float* __restrict__ call, float* __restrict__ put) {
+    pdl_enter();
+    const int64_t n4 = n >> 2;
+    const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
+    sweep_groups(reinterpret_cast<const float4*>(S), reinterpret_cast<const float4*>(X),
+                 reinterpret_cast<const float4*>(T), blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x,
+                 n4, stride, [&](int64_t i, const float4& s, const float4& x, const float4& t) {
+                     float4 cv, pv;
+                     price4(s, x, t, c, cv, pv);
+                     st_stream_f4(reinterpret_cast<float4*>(call) + i, cv);
+                     st_stream_f4(reinterpret_cast<float4*>(put) + i, pv);
+                 });
     // ragged tail (n % 4 elements)
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (n & 3)) {
         const int64_t e = (n4 << 2) + threadIdx.x;
@@ -147,27 +208,24 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
                                                          double2* __restrict__ partial) {
     __shared__ double2 s_part[8];
     __shared__ int s_last;
-    // per-thread partials in fp32 (a thread prices ~n/(grid*256) options), fp64 from the warp up
-    float fc = 0.f, fp = 0.f;
+    pdl_enter();
+    // per-thread partials of w and u in fp32 (a thread prices ~n/(grid*256) options), fp64 from
+    // the warp up; sum call = sum w + sum u / 2, sum put = sum w - sum u / 2 (price2_wu)
+    float2 aw = make_float2(0.f, 0.f), au = make_float2(0.f, 0.f);
     const int64_t n4 = n >> 2;
     const int64_t stride = static_cast<int64_t>(gridDim.x) * blockDim.x;
-    const float4* S4 = reinterpret_cast<const float4*>(S);
-    const float4* X4 = reinterpret_cast<const float4*>(X);
-    const float4* T4 = reinterpret_cast<const float4*>(T);
-    int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x;
-    float4 s, x, t;
-    if (i < n4) { s = ld_stream_f4(S4 + i); x = ld_stream_f4(X4 + i); t = ld_stream_f4(T4 + i); }
-    for (; i < n4; i += stride) {
-        const int64_t nx = i + stride;
-        float4 s2 = s, x2 = x, t2 = t;
-        if (nx < n4) { s2 = ld_stream_f4(S4 + nx); x2 = ld_stream_f4(X4 + nx); t2 = ld_stream_f4(T4 + nx); }
-        float4 cv, pv;
-        price4(s, x, t, c, cv, pv);
-        fc += (cv.x + cv.y) + (cv.z + cv.w);
-        fp += (pv.x + pv.y) + (pv.z + pv.w);
-        s = s2; x = x2; t = t2;
-    }
-    double ac = fc, ap = fp;
+    sweep_groups(reinterpret_cast<const float4*>(S), reinterpret_cast<const float4*>(X),
+                 reinterpret_cast<const float4*>(T), blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x,
+                 n4, stride, [&](int64_t, const float4& s, const float4& x, const float4& t) {
+                     float2 w0, u0, w1, u1;
+                     price2_wu(make_float2(s.x, s.y), make_float2(x.x, x.y), make_float2(t.x, t.y), c, w0, u0);
+                     price2_wu(make_float2(s.z, s.w), make_float2(x.z, x.w), make_float2(t.z, t.w), c, w1, u1);
+                     aw = add2(aw, add2(w0, w1));
+                     au = add2(au, add2(u0, u1));
+                 });
+    const double w = static_cast<double>(aw.x) + static_cast<double>(aw.y);
+    const double hu = 0.5 * (static_cast<double>(au.x) + static_cast<double>(au.y));
+    double ac = w + hu, ap = w - hu;
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x < (n & 3)) {
         const int64_t e = (n4 << 2) + threadIdx.x;
         float cv, pv;
@@ -182,7 +240,7 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
     __syncthreads();
     if (threadIdx.x == 0) {
         double2 b = s_part[0];
-        for (int w = 1; w < (blockDim.x >> 5); ++w) { b.x += s_part[w].x; b.y += s_part[w].y; }
+        for (int k = 1; k < (blockDim.x >> 5); ++k) { b.x += s_part[k].x; b.y += s_part[k].y; }
         __stcg(partial + blockIdx.x, b);
         __threadfence();
         s_last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
@@ -215,6 +273,9 @@ static Consts make_consts(float r, float sigma) {
     c.inv_sigma = 1.0f / sigma;
     c.sigma = sigma;
     c.neg_r_log2e = -r * 1.44269504088896341f;
+    c.a_l2 = static_cast<float>((static_cast<double>(r) + 0.5 * sigma * static_cast<double>(sigma)) * 1.4426950408889634);
+    c.b_l2 = static_cast<float>((static_cast<double>(r) - 0.5 * sigma * static_cast<double>(sigma)) * 1.4426950408889634);
+    c.ln2_over_sigma = static_cast<float>(0.6931471805599453 / sigma);
     return c;
 }
 
@@ -236,8 +297,7 @@ cudaError_t launch_map(const float* S, const float* X, const float* T, int64_t n
                        float* call, float* put, cudaStream_t stream) {
     if (n == 0) return cudaSuccess;
     const int grid = grid_for(reinterpret_cast<const void*>(&map_kernel), n);
-    map_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), call, put);
-    return cudaGetLastError();
+    return launch_pdl(&map_kernel, dim3(grid), dim3(256), 0, stream, S, X, T, n, make_consts(r, sigma), call, put);
 }
 
 cudaError_t launch_map_reduce(const float* S, const float* X, const float* T, int64_t n, float r,
@@ -246,8 +306,8 @@ cudaError_t launch_map_reduce(const float* S, const float* X, const float* T, in
     if (grid > red::kMaxCtas) grid = red::kMaxCtas;
     unsigned* ticket = static_cast<unsigned*>(ws);
     double2* partial = reinterpret_cast<double2*>(static_cast<char*>(ws) + 256);
-    map_reduce_kernel<<<grid, 256, 0, stream>>>(S, X, T, n, make_consts(r, sigma), sums, ticket, partial);
-    return cudaGetLastError();
+    return launch_pdl(&map_reduce_kernel, dim3(grid), dim3(256), 0, stream, S, X, T, n, make_consts(r, sigma), sums,
+                      ticket, partial);
 }
 
 }  // namespace bs

@@ -172,4 +172,32 @@ __host__ __device__ constexpr T mn(T a, T b) { return b < a ? b : a; }
 template <typename T>
 __host__ __device__ constexpr T mx(T a, T b) { return a < b ? b : a; }
 
+// ---------------------------------------------------------------- programmatic dependent launch
+// Streaming kernels are launched with programmatic stream serialization: the next launch on the
+// stream may be scheduled while this grid drains, so its CTAs are resident when the SMs free up
+// instead of after a full launch round trip. pdl_enter() is the first statement of such a kernel:
+// griddepcontrol.wait returns only once every prerequisite grid has COMPLETED and its memory is
+// visible, so the kernel never reads anything an earlier launch is still writing (the stream-order
+// semantics are unchanged); it then allows its own dependents to be scheduled.
+__device__ __forceinline__ void pdl_enter() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+bool pdl_enabled();   // false when LIME_NO_PDL is set in the environment (A/B and debugging)
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
+                              Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 }  // namespace lime

@@ -98,6 +98,7 @@ __global__ void __launch_bounds__(256) reduce_kernel(const T* __restrict__ x, in
     using A = typename P::Acc;
     constexpr int V = 16 / sizeof(T);   // elements per 128-bit load
     A* partial = static_cast<A*>(partial_raw);
+    pdl_enter();
     __shared__ A s_warp[8];
     __shared__ int s_last;
 
@@ -186,8 +187,8 @@ static cudaError_t launch_t(const void* x, int64_t n, void* out, void* ws, cudaS
     if (grid > kMaxCtas) grid = kMaxCtas;
     unsigned* ticket = static_cast<unsigned*>(ws);
     void* partial = static_cast<char*>(ws) + 256;
-    reduce_kernel<OP, T><<<grid, block, 0, stream>>>(static_cast<const T*>(x), n, static_cast<T*>(out), ticket, partial);
-    return cudaGetLastError();
+    return launch_pdl(&reduce_kernel<OP, T>, dim3(grid), dim3(block), 0, stream, static_cast<const T*>(x), n,
+                      static_cast<T*>(out), ticket, partial);
 }
 
 cudaError_t launch(Op op, Dt dt, const void* x, int64_t n, void* out, void* ws, cudaStream_t stream) {

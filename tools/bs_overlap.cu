@@ -9,6 +9,7 @@
 namespace lime {
 const LaunchOverride& launch_override() { static LaunchOverride o; return o; }
 int device_num_sms() { return 148; }
+bool pdl_enabled() { return true; }
 namespace red { }
 }
 using namespace lime;
