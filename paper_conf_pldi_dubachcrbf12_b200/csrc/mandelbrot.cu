@@ -6,8 +6,8 @@
 // compiled SASS keeps it that way.
 //
 // B200 design (DESIGN.md §"Mandelbrot"):
-//  * A5/A6c: each lane iterates TWO horizontally adjacent pixels with packed FMUL2/FADD2
-//    (8 packed ops per pixel pair per iteration instead of 16 scalar ones).
+//  * A5/A6c: each lane iterates TWO horizontally adjacent pixels with packed FFMA2
+//    (7 packed ops per pixel pair per iteration instead of 16 scalar ones).
 //  * Branch-free iteration with sticky "alive" predicates; the warp checks __any_sync once
 //    per 16 unrolled iterations, so escaped lanes cost at most 15 extra iterations.
 //  * A1: persistent CTAs pull 16x4-pixel warp tiles from a global atomic queue (dynamic
@@ -35,14 +35,16 @@ struct Args {
 };
 
 // Every binary32 op is written as ONE fused multiply-add whose extra operand makes it exact:
-//   a*b = fma(a, b, -0),  a+b = fma(a, 1, b),  a-b = fma(b, -1, a)
+//   a*b = fma(a, b, -0),  a+b = fma(a, 1, b),  a-b = fma(b, -1, a),  (a+a)+c = fma(a, 2, c)
+// (the last: a+a = 2a is exact, so R7's two roundings of 2xy + cy collapse into the fma's one;
+// 7 packed ops per iteration instead of 8)
 // ptxas contracts packed mul.rn/add.rn.f32x2 pairs into FFMA2 even with --fmad=false (observed
 // on CUDA 12.9, see tests/test_sass_guards.py), which changes rounding; an FFMA2 cannot be
 // contracted further, so this spelling keeps one IEEE rounding per operation of R7.
 // n += alive as ONE predicated integer add per pixel: the sticky FSETP.LE.AND's predicate guards
 // the add directly (the C++ spellings `n += a`, `if (a) n++` compile to two IADD3 per pixel on
-// CUDA 12.9, and this loop is issue-bound: 8 packed FP32 ops = 16 pipe cycles per iteration
-// against ~15 issued instructions).
+// CUDA 12.9, and this loop is issue-bound: 7 packed FP32 ops = 14 pipe cycles per iteration
+// against ~12 issued instructions).
 __device__ __forceinline__ void count(int& n, bool alive) {
     asm("{ .reg .pred p; setp.ne.b16 p, %1, 0; @p add.s32 %0, %0, 1; }" : "+r"(n) : "h"(static_cast<short>(alive)));
 }
@@ -62,7 +64,8 @@ struct State {
         count(n1, a1);
         const float2 xy = fma2(x, y, z);
         x = fma2(fma2(yy, mone, xx), one, cx);       // x <- (x^2 - y^2) + cx
-        y = fma2(fma2(xy, one, xy), one, cy);        // y <- (xy + xy) + cy
+        y = fma2(xy, bcast2(2.0f), cy);              // y <- (xy + xy) + cy: xy + xy = 2 xy is exact, so
+                                                     // fma(xy, 2, cy) = rn(2 xy + cy) rounds once, as R7
     }
 };
 

@@ -60,3 +60,17 @@ def test_fused_sums(lime, n):
     assert abs(sums[1] - sp) <= BS_TOL * max(abs(sp), 1.0)
     again = lime.map_reduce_blackscholes_sum(_dev(S), _dev(X), _dev(T), float(R), float(SIG)).cpu().numpy()
     assert np.array_equal(sums, again)                               # deterministic, ws self-resets
+
+
+@pytest.mark.parametrize("k", range(8))
+def test_fused_single_option_tails(lime, k):
+    # the fused kernel's element (sums of w = A - B and u = S - K; call = w + u/2, put = w - u/2)
+    # on one tail option at a time, padded to a multiple of 4 with copies so the vector path runs
+    S = np.array([5, 30, 5, 30, 100, 1, 50, 50], dtype=np.float32)
+    X = np.array([100, 1, 90, 2, 1, 100, 50, 50], dtype=np.float32)
+    T = np.array([0.25, 0.25, 10, 10, 0.01, 0.01, 0.0001, 50], dtype=np.float32)
+    s, x, t = (np.repeat(a[k:k + 1], 8) for a in (S, X, T))
+    sums = lime.map_reduce_blackscholes_sum(_dev(s), _dev(x), _dev(t), float(R), float(SIG)).cpu().numpy()
+    sc, sp = oracle.blackscholes_sums(s, x, t, R, SIG)
+    assert abs(sums[0] - sc) <= BS_TOL * max(abs(sc), 8.0)       # per option: 1e-5 * max(|price|, 1)
+    assert abs(sums[1] - sp) <= BS_TOL * max(abs(sp), 8.0)

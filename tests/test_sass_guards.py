@@ -33,11 +33,12 @@ def _fn(sass, pat):
 
 
 def test_mandelbrot_has_no_inexact_fma(sass):
-    # R7 bit-exactness: every FFMA/FFMA2 in the Mandelbrot kernel must be an exact rewrite of a
-    # single op (multiplier +-1 immediate), never a contracted x*y+z.
+    # R7 bit-exactness: every FFMA/FFMA2 in the Mandelbrot kernel must be an exact rewrite of
+    # R7's ops (multiplier +-1 immediate: one add/sub; multiplier 2: (a + a) + c, where a + a is
+    # exact so R7's two roundings equal the fma's one), never a contracted x*y+z.
     for ins in _fn(sass, r"mandel"):
         if re.match(r"(@!?P\d )?FFMA", ins):
-            assert re.search(r",\s*-?1(\.0+)?\s*,", ins), ins
+            assert re.search(r",\s*(-?1|2)(\.0+)?\s*,", ins), ins
 
 
 def test_mandelbrot_uses_packed_fp32(sass):
