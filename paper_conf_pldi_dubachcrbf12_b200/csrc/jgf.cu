@@ -137,8 +137,23 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
         const int step_u = p;                         // R n mod m
         int q = 0;                                    // R n u mod m
         T a = 0, b = 0;
+        // fp64: g_{Ru+v} for the next u is loaded one iteration ahead (the constant-bank loads at a
+        // run-time offset otherwise stall the first DFMA of each chain; 46.4 -> 42.0 us). fp32 is
+        // faster without it (24.7 vs 27.6 us: 64-register cap), profiles/experiments/jg_series_variants_r01m.jsonl.
+        constexpr bool kAhead = sizeof(T) == 8;
+        T gn[R];
+#pragma unroll
+        for (int v = 0; v < R; ++v) gn[v] = kAhead ? G.g[v] : T(0);
 #pragma unroll 1
         for (int u = 0; u < NU; ++u) {
+            T g[R];
+#pragma unroll
+            for (int v = 0; v < R; ++v) g[v] = kAhead ? gn[v] : G.g[u * R + v];
+            if constexpr (kAhead) {
+                const int un = u + 1 < NU ? u + 1 : u;
+#pragma unroll
+                for (int v = 0; v < R; ++v) gn[v] = G.g[un * R + v];
+            }
             const T ur = sc[q], ui = ss[q];
             q += step_u;
             q -= (q >= kSeriesM) ? kSeriesM : 0;
@@ -146,8 +161,8 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
             w0.x = w0.y = w1.x = w1.y = 0;
 #pragma unroll
             for (int v = 0; v < R; ++v) {
-                if (v & 1) w1 = cfma(G.g[u * R + v], V[v], w1);
-                else       w0 = cfma(G.g[u * R + v], V[v], w0);
+                if (v & 1) w1 = cfma(g[v], V[v], w1);
+                else       w0 = cfma(g[v], V[v], w0);
             }
             const T wr = w0.x + w1.x, wi = w0.y + w1.y;
             a = fma(ur, wr, a);

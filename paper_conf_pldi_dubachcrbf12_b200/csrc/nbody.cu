@@ -454,6 +454,7 @@ __global__ void __launch_bounds__(16 * kMaxSplitsSmall) force_small_kernel(const
     float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
     __shared__ __align__(8) uint64_t bar[kMaxSplitsSmall / 2];
 
+    pdl_enter();
     const int warp = threadIdx.x >> 5;
     const unsigned lane = lane_id();
     const SmallLane sl;
@@ -508,8 +509,8 @@ static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
         attr = kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16;
     }
     const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
-    force_small_kernel<<<static_cast<unsigned>(ctas), 32 * ceil_div(a.splits, 2), smem, stream>>>(a);
-    return cudaGetLastError();
+    return launch_pdl(&force_small_kernel, dim3(static_cast<unsigned>(ctas)), dim3(32 * ceil_div(a.splits, 2)), smem,
+                      stream, a);
 }
 
 // =====================================================================================
@@ -911,6 +912,7 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
 // ------------------------------------------------------------------------ integrator (A9)
 __global__ void __launch_bounds__(256) integrate_kernel(float4* __restrict__ pos, float4* __restrict__ vel,
                                                         const float4* __restrict__ accel, int64_t n, float dt) {
+    pdl_enter();
     for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n;
          i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
         const float4 a = ld_stream_f4(accel + i);
@@ -932,8 +934,7 @@ cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int6
     if (n == 0) return cudaSuccess;
     int grid = launch_override().grid_ctas;
     if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(n, 256), 8LL * device_num_sms()));
-    integrate_kernel<<<grid, 256, 0, stream>>>(pos, vel, accel, n, dt);
-    return cudaGetLastError();
+    return launch_pdl(&integrate_kernel, dim3(grid), dim3(256), 0, stream, pos, vel, accel, n, dt);
 }
 
 }  // namespace nbody

@@ -17,7 +17,8 @@ KEYMAP = {"nbody1m": "nbody_force_1m", "nbody1m_p8": "nbody_force_1m_p8", "nbody
 
 def main(tag):
     out = os.path.join(ROOT, "gpurun_out")
-    prof = os.path.join(ROOT, "profiles")
+    prof = os.environ.get("PROF_DIR") or os.path.join(ROOT, "profiles")   # PROF_DIR: summarise on the GPU box
+    os.makedirs(prof, exist_ok=True)
     summary, traffic = {}, {}
     for k, name in KEYMAP.items():
         rep = os.path.join(out, f"prof_{k}_{tag}.ncu-rep")
