@@ -549,7 +549,11 @@ def run_extras(peaks, flush):
     out["jg_crypt"] = {"workload": "F4: JG-Crypt IDEA-ECB over 3 MiB (Table 3)", "value": data.numel() / (med * 1e-3),
                        "unit": "bytes/s", "ms_per_launch": med,
                        "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
-                                    "traffic": None, "note": "3 MiB is latency-bound: one wave of 148 x 8 CTAs"}}
+                                    "traffic": None,
+                                    "note": "not HBM-bound at 3 MiB (6 MB of traffic = 1 us at HBM speed): integer-issue-bound "
+                                            "(ncu r01n: issue active 78 %; 333 SASS instructions per 8-byte block, 34 "
+                                            "multiplications mod 2^16+1), one wave of 768 CTAs; ~6 us of the event-timed "
+                                            "launch is the launch floor (tools/launch_floor.py)"}}
     del data, enc
 
     # reduction `!`: sum over 2^28 fp32 (1 GiB)

@@ -202,27 +202,31 @@ struct IdeaKeys {
 };
 
 __device__ __forceinline__ uint32_t idea_mul(uint32_t a, uint32_t b) {
-    // a * b mod (2^16 + 1) on 16-bit operands where 0 stands for 2^16
+    // a * b mod (2^16 + 1) on 16-bit operands where 0 stands for 2^16. Only the low 16 bits of a
+    // are significant (the callers leave sums unmasked), b is a clean sub-key; the result's low 16
+    // bits are the product (bit 16 may be set: p mod 65537 = 65536 stands for 0 mod 2^16). For a, b
+    // nonzero p mod 65537 is never 0 (65537 is prime) and the constant-divisor remainder is
+    // IMAD.HI + SHF + IMAD; p = 0 exactly when a or b is 2^16, where the product is 1 - a - b.
+    a &= 0xFFFFu;
     const uint32_t p = a * b;
-    const uint32_t lo = p & 0xFFFFu, hi = p >> 16;
-    const uint32_t r = lo - hi + (lo < hi ? 1u : 0u);
-    return (p != 0u ? r : (1u - a - b)) & 0xFFFFu;
+    return p != 0u ? p % 65537u : 1u - a - b;
 }
 
 __device__ __forceinline__ uint2 idea_block(uint2 v, const IdeaKeys& k) {
-    // bytes b0..b7 of the block; words are big-endian (R15)
+    // bytes b0..b7 of the block; words are big-endian (R15). Words are kept modulo 2^16 lazily: only
+    // their low 16 bits are significant, idea_mul masks its data operand, the output takes low bytes.
     uint32_t x1 = __byte_perm(v.x, 0, 0x4401), x2 = __byte_perm(v.x, 0, 0x4423);
     uint32_t x3 = __byte_perm(v.y, 0, 0x4401), x4 = __byte_perm(v.y, 0, 0x4423);
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
         const uint32_t* z = k.z + 6 * r;
         x1 = idea_mul(x1, z[0]);
-        x2 = (x2 + z[1]) & 0xFFFFu;
-        x3 = (x3 + z[2]) & 0xFFFFu;
+        x2 = x2 + z[1];
+        x3 = x3 + z[2];
         x4 = idea_mul(x4, z[3]);
         const uint32_t t0 = idea_mul(x1 ^ x3, z[4]);
-        const uint32_t t1 = idea_mul((t0 + (x2 ^ x4)) & 0xFFFFu, z[5]);
-        const uint32_t t2 = (t0 + t1) & 0xFFFFu;
+        const uint32_t t1 = idea_mul(t0 + (x2 ^ x4), z[5]);
+        const uint32_t t2 = t0 + t1;
         x1 ^= t1;
         x4 ^= t2;
         const uint32_t a = x2 ^ t2;
@@ -230,8 +234,8 @@ __device__ __forceinline__ uint2 idea_block(uint2 v, const IdeaKeys& k) {
         x3 = a;
     }
     const uint32_t y1 = idea_mul(x1, k.z[48]);
-    const uint32_t y2 = (x3 + k.z[49]) & 0xFFFFu;
-    const uint32_t y3 = (x2 + k.z[50]) & 0xFFFFu;
+    const uint32_t y2 = x3 + k.z[49];
+    const uint32_t y3 = x2 + k.z[50];
     const uint32_t y4 = idea_mul(x4, k.z[51]);
     // back to bytes: word w -> (hi byte, lo byte)
     return make_uint2(__byte_perm(y1, y2, 0x4501), __byte_perm(y3, y4, 0x4501));
