@@ -13,6 +13,8 @@
 //               accumulator in TMEM), tcgen05.commit releases smem stages / publishes accumulators
 //   warps 2..5  epilogue: tcgen05.ld TMEM -> registers -> fp32 C (A7), double-buffered TMEM
 //               accumulators (2 x 256 columns) so the epilogue of tile t overlaps the MMAs of t+1.
+#include <cstring>
+
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -246,7 +248,10 @@ constexpr int STAGES = 6;
 constexpr uint32_t kStageA = BM * BK * 2;            // 16 KB
 constexpr uint32_t kStageB = (BN / 2) * BK * 2;      // 16 KB
 constexpr uint32_t kStageBytes = kStageA + kStageB;
-constexpr size_t kSmemBytes = 1024 + STAGES * kStageBytes + 256;
+// epilogue staging for TMA stores: per epilogue warp two 32 x 32 fp32 boxes (4 KB each, 128B-swizzled)
+constexpr uint32_t kEpiBox = 32 * 32 * 4;
+constexpr uint32_t kEpiBytes = 4 * 2 * kEpiBox;
+constexpr size_t kSmemBytes = 1024 + STAGES * kStageBytes + kEpiBytes + 256;
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(BN >> 3) << 17) |
                             (static_cast<uint32_t>(256 >> 4) << 24);
 }  // namespace two
@@ -275,8 +280,22 @@ __device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
                  :: "r"(smem_addr(bar)), "h"(static_cast<uint16_t>(3)) : "memory");
 }
 
+// TMA tensor store of one smem box (bulk-group completion; no mbarrier)
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* src, int c0, int c1) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                 :: "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_addr(src)) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(N) : "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void st_shared_f4(uint32_t addr, float a, float b, float c, float d) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" :: "r"(addr), "f"(a), "f"(b), "f"(c), "f"(d) : "memory");
+}
+
 struct Params2 {
     float* C;
+    int tma_store;             // 1: C is written through tmap_c (N % 4 == 0, 16-B aligned C)
     int M, N, K;
     int group;                 // raster group: pair-tile rows that sweep the N tiles together
     int num_m, num_n, num_k;   // num_m counts 256-row pair tiles
@@ -296,10 +315,11 @@ __device__ __forceinline__ void tile_coords2(int t, const Params2& p, int& mb, i
 
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
-             const __grid_constant__ Params2 p) {
+             const __grid_constant__ CUtensorMap tmap_c, const __grid_constant__ Params2 p) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + two::STAGES * two::kStageBytes);
+    uint8_t* epi = smem + two::STAGES * two::kStageBytes;                 // 1024-B aligned staging
+    uint64_t* full = reinterpret_cast<uint64_t*>(epi + two::kEpiBytes);
     uint64_t* empty = full + two::STAGES;
     uint64_t* tfull = empty + two::STAGES;
     uint64_t* tempty = tfull + 2;
@@ -315,6 +335,7 @@ gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__
     if (warp == 0 && lane == 0) {
         prefetch_tmap(&tmap_a);
         prefetch_tmap(&tmap_b);
+        if (p.tma_store) prefetch_tmap(&tmap_c);
         for (int s = 0; s < two::STAGES; ++s) {
             mbar_init(&full[s], 1);      // leader's producer arms it with both CTAs' tx bytes
             mbar_init(&empty[s], 1);     // released by the leader's MMA commit (multicast to both CTAs)
@@ -398,6 +419,36 @@ gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__
             const uint32_t tbase = tmem_base + (static_cast<uint32_t>(quad * 32) << 16) + static_cast<uint32_t>(acc * two::BN);
             float* crow = p.C + static_cast<int64_t>(row) * p.N;
             const bool vec_ok = (p.N & 3) == 0;
+            if (p.tma_store) {
+                // TMEM -> registers -> this warp's 128B-swizzled 32 x 32 smem box -> one TMA store of
+                // full 128-byte lines (the direct path writes each row's 16-byte pieces from 32 lanes:
+                // 8x the L2 write requests); two boxes in turn, a box is rewritten only after the
+                // store issued from it two chunks earlier has read it. The store clips at M and N.
+                const uint32_t box0 = smem_addr(epi + (quad * 2) * two::kEpiBox);
+                const int row0 = mb * 256 + static_cast<int>(rank) * two::BM + quad * 32;
+#pragma unroll 1
+                for (int c = 0; c < two::BN; c += 32) {
+                    float v[32];
+                    tmem_ld32(tbase + c, v);
+                    const uint32_t box = box0 + static_cast<uint32_t>(((c >> 5) & 1) * two::kEpiBox);
+                    if (lane == 0) bulk_wait_read<1>();
+                    __syncwarp();
+#pragma unroll
+                    for (int q = 0; q < 8; ++q)
+                        st_shared_f4(box + static_cast<uint32_t>(lane * 128 + ((q ^ (lane & 7)) << 4)), v[4 * q],
+                                     v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+                    fence_proxy_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        tma_store_2d(&tmap_c, epi + (box - smem_addr(epi)), nb * two::BN + c, row0);
+                        bulk_commit();
+                    }
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cluster(tempty_leader0 + static_cast<uint32_t>(acc * 8));
+                continue;
+            }
 #pragma unroll 1
             for (int c = 0; c < two::BN; c += 32) {
                 float v[32];
@@ -420,6 +471,7 @@ gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__
             __syncwarp();
             if (lane == 0) mbar_arrive_cluster(tempty_leader0 + static_cast<uint32_t>(acc * 8));
         }
+        if (p.tma_store && lane == 0) bulk_wait_all();   // staging smem must outlive the stores
     }
 
     tc_fence_before();
@@ -455,6 +507,18 @@ static bool make_map(CUtensorMap* map, const void* base, uint64_t rows, uint64_t
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// C [M][N] fp32 for the epilogue's TMA stores: 32 x 32 boxes (128-byte rows), 128B swizzle
+static bool make_map_c(CUtensorMap* map, void* base, uint64_t rows, uint64_t cols) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[2] = {cols, rows};
+    const cuuint64_t strides[1] = {cols * 4};
+    const cuuint32_t box[2] = {32, 32};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+              CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
                         cudaStream_t stream) {
     const LaunchOverride& ov = launch_override();
@@ -472,6 +536,10 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
         p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
         p.num_tiles = p.num_m * p.num_n;
         p.group = ov.block_threads > 0 ? ov.block_threads : 8;   // override: raster group (sweep)
+        CUtensorMap mc;
+        std::memset(&mc, 0, sizeof mc);
+        p.tma_store = ((N & 3) == 0 && (reinterpret_cast<uintptr_t>(C) & 15) == 0 && ov.per_thread != 3 &&
+                       make_map_c(&mc, C, M, N)) ? 1 : 0;
         static bool attr2 = false;
         if (!attr2) {
             cudaError_t e = cudaFuncSetAttribute(gemm2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -481,7 +549,7 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
         }
         int clusters = ov.grid_ctas > 0 ? mx(1, ov.grid_ctas / 2) : device_num_sms() / 2;
         clusters = mn(clusters, p.num_tiles);
-        gemm2_kernel<<<2 * clusters, kThreads, two::kSmemBytes, stream>>>(ma, mb, p);
+        gemm2_kernel<<<2 * clusters, kThreads, two::kSmemBytes, stream>>>(ma, mb, mc, p);
         return cudaGetLastError();
     }
     if (!make_map(&ma, A, M, K, BM) || !make_map(&mb, Bt, N, K, BN)) return cudaErrorInvalidValue;
