@@ -1,5 +1,6 @@
-"""A/B the 2-CTA GEMM epilogue at 8192^3: TMA-store epilogue (default) vs direct st.global
-(launch override per_thread=3); cuBLAS fp32-out beside. One JSON line per variant."""
+"""A/B the 2-CTA GEMMs at 8192^3: 256x256 pair tile with the TMA-store epilogue (default) or direct
+st.global (per_thread=3); cuBLAS fp32-out beside. One JSON line per variant. (The 512x256 wide pair
+tile measured with it is recorded in profiles/experiments/gemm_wide_pair_tma_store_r01n.diff.txt.)"""
 import json
 import os
 import sys
@@ -21,8 +22,8 @@ C = torch.empty((M, M), device="cuda")
 with lime.launch_override(per_thread=3):
     ref = lime.map_matmul_bf16(A, B).clone()
 for rep in range(2):
-    for pt, name in ((0, "tma_store"), (3, "st_global")):
-        with lime.launch_override(per_thread=pt):
+    for pt, g, name in ((0, 0, "pair256_tma_store"), (3, 0, "pair256_st_global")):
+        with lime.launch_override(per_thread=pt, block_threads=g):
             ms = time_launches(lambda: lime.map_matmul_bf16(A, B, C), 20, 3, flush, writes_output=True)[0]
         print(json.dumps({"variant": name, "ms": ms, "TF": 2 * M**3 / ms / 1e9, "identical": bool(torch.equal(C, ref))}),
               flush=True)
