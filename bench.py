@@ -311,13 +311,7 @@ def run_nbody(args, rank, world, local):
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"BASELINE.json configs[4]: N-body all-pairs {n} bodies fp32, index-space "
-                                   "sharded, NCCL all-gather per step",
-                       "n_bodies": n, "eps2": EPS2, "dt": DT, "targets_per_gpu": sim.count,
-                       "parallelism": f"target-index shards x{world}" + (" + all_gather" if world > 1 else ""),
-                       "l2": "flushed before every step inside the timed region (2x L2 write); the 16 MiB source "
-                             "array is then re-read from L2 by design (broadcast operand)",
-                       "inputs": "inputs.nbody_bodies(seed=5): U[-1,1)^3, m=1/N, v0=0"},
+            "config": headline_config(n, world),
             "roofline": roofline, "e2e": e2e, "gpu_launches": (4 if n > 8192 else 2) * args.steps + (args.steps if world > 1 else 0), "clocks": clk,
             "momentum_residual": float(mom.norm().item())}
     return line
@@ -665,6 +659,18 @@ def oracle_beside(configs: dict) -> None:
         put("reduce_sum_f32", float(1 << 26), sec, "2^26 of the 2^28 elements")
 
 
+def headline_config(n, world):
+    """The headline workload's config, shared by both arms (the reference arm times a bounded oracle
+    sample of this same workload, described in its cpu_baseline.sample)."""
+    return {"workload": f"BASELINE.json configs[4]: N-body all-pairs {n} bodies fp32, index-space "
+                        "sharded, NCCL all-gather per step",
+            "n_bodies": n, "eps2": EPS2, "dt": DT, "targets_per_gpu": n // world,
+            "parallelism": f"target-index shards x{world}" + (" + all_gather" if world > 1 else ""),
+            "l2": "flushed before every step inside the timed region (2x L2 write); the 16 MiB source "
+                  "array is then re-read from L2 by design (broadcast operand)",
+            "inputs": "inputs.nbody_bodies(seed=5): U[-1,1)^3, m=1/N, v0=0"}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return None
@@ -689,7 +695,7 @@ def run_reference(args, rank, world):
     return {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": per_step * 1e3, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
-            "config": {"workload": "BASELINE.json configs[4]: N-body 2^20 bodies (oracle sample)", "n_bodies": n},
+            "config": headline_config(n, world),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 

@@ -27,7 +27,8 @@ def _check(C, A, Bt, rows=None, cols=None):
 
 
 @pytest.mark.parametrize("M,N,K", [(128, 256, 64), (1, 1, 8), (33, 47, 72), (300, 520, 200), (256, 512, 1024),
-                                   (1000, 1000, 1000), (8192 // 8, 64, 128), (129, 257, 4104)])
+                                   (1000, 1000, 1000), (8192 // 8, 64, 128), (129, 257, 4104),
+                                   (300, 517, 64), (513, 1030, 136)])
 def test_matmul_small_matches_oracle(lime, M, N, K):
     A, Bt = inputs.matmul_operands(M, N, K, seed=M + N + K)
     C = lime.map_matmul_bf16(_bf(A), _bf(Bt)).cpu().numpy()
@@ -68,3 +69,16 @@ def test_matmul_launch_independent(lime):
     for g in (1, 7, 64):
         with lime.launch_override(grid_ctas=g):
             assert torch.equal(lime.map_matmul_bf16(_bf(A), _bf(Bt)), C0)
+
+
+@pytest.mark.parametrize("M,N,K", [(300, 520, 200), (1024, 1024, 512), (513, 1028, 136)])
+def test_matmul_epilogue_forms_identical(lime, M, N, K):
+    # the 2-CTA kernel's TMA-store epilogue (default for N % 4 == 0) and its direct st.global form
+    # (launch override per_thread=3; the path N % 4 != 0 takes) write the same bits, ragged M/N included
+    A, Bt = inputs.matmul_operands(M, N, K, seed=M + 3 * N + K)
+    C_tma = lime.map_matmul_bf16(_bf(A), _bf(Bt))
+    with lime.launch_override(per_thread=3):
+        C_st = lime.map_matmul_bf16(_bf(A), _bf(Bt))
+    assert torch.equal(C_tma, C_st)
+    e, fro = _check(C_tma.cpu().numpy(), A, Bt)
+    assert e <= MATMUL_RTOL and fro <= MATMUL_RTOL
