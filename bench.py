@@ -447,9 +447,12 @@ def run_extras(peaks, flush):
         med, _ = time_launches(lambda: lime.map_matmul_bf16(A, Bt, Cm), 20, 3, flush, writes_output=True)
         tf = 2.0 * M * N * K / (med * 1e-3) / 1e12
         cub, _ = time_launches(lambda: torch.matmul(A, Bt.t()), 20, 3, flush, writes_output=True)
+        # cuBLAS with this kernel's own output type (fp32 C), the like-for-like library baseline
+        cub32, _ = time_launches(lambda: torch.mm(A, Bt.t(), out_dtype=torch.float32), 20, 3, flush, writes_output=True)
         out["matmul"] = {"workload": "configs[3]: matmul 8192^3 bf16 in, fp32 accumulate/out (tcgen05)",
                          "value": M * N / (med * 1e-3), "unit": "dot products/s", "ms_per_launch": med,
-                         "tflops": tf, "cublas_bf16_out_ms": cub,
+                         "tflops": tf, "cublas_bf16_out_ms": cub, "cublas_fp32_out_ms": cub32,
+                         "vs_cublas_fp32_out": cub32 / med,
                          "roofline": {"bound": "tensor", "achieved": tf, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
                                       "frac": tf / peaks["bf16_tflops"], "traffic": ncu_traffic("matmul")}}
         del A, Bt, Cm
