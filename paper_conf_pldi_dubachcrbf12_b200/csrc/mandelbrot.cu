@@ -9,8 +9,8 @@
 //  * A5/A6c: each lane iterates TWO horizontally adjacent pixels with packed FFMA2
 //    (7 packed ops per pixel pair per iteration instead of 16 scalar ones).
 //  * Branch-free iteration with sticky "alive" predicates; the warp checks __any_sync once
-//    per 16 unrolled iterations, so escaped lanes cost at most 15 extra iterations.
-//  * A1: persistent CTAs pull 16x4-pixel warp tiles from a global atomic queue (dynamic
+//    per 32 unrolled iterations, so escaped lanes cost at most 31 extra iterations.
+//  * A1: persistent CTAs pull 8x8-pixel warp tiles from a global atomic queue (dynamic
 //    load balance: escape times vary by 1000x across the frame); the last warp to finish
 //    resets the queue (self-cleaning workspace).
 #include "common.cuh"
@@ -163,7 +163,10 @@ cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t
         case 4: return launch_t<8, 8>(a, stream);
         case 5: return launch_t<16, 16>(a, stream);
         case 6: return launch_t<8, 32>(a, stream);
-        default: return launch_t<8, 16>(a, stream);
+        case 7: return launch_t<4, 32>(a, stream);
+        case 8: return launch_t<8, 64>(a, stream);
+        case 1: return launch_t<8, 16>(a, stream);
+        default: return launch_t<4, 32>(a, stream);   // = case 7 (tools/tune_mandel.py: 3.19 vs 3.22 ms for 16x4/16)
     }
 }
 
