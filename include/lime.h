@@ -26,7 +26,12 @@
  * Streams. `stream` is a cudaStream_t passed as void* (NULL = legacy default
  *   stream). All work is enqueued asynchronously on it; the library never
  *   synchronises, except `_host` entry points, which synchronise `stream`
- *   before returning (their outputs are host memory).
+ *   before returning (their outputs are host memory). The streaming kernels
+ *   (Black-Scholes, reductions, the small N-Body map, the integrator) are
+ *   launched with programmatic dependent launch: their first instruction waits
+ *   until every earlier grid on the stream has completed and its writes are
+ *   visible, so stream order is unchanged; only the launch itself overlaps the
+ *   previous grid's drain. Setting LIME_NO_PDL in the environment disables it.
  * Workspaces. Entry points taking (ws, ws_bytes) need a device scratch buffer
  *   of at least the size returned by the matching *_workspace_bytes() query,
  *   ZERO-FILLED before its first use; every call leaves every word a later
@@ -184,16 +189,22 @@ lime_status lime_nbody_simulate_host(float *h_pos, float *h_vel, int64_t n, int3
  * no overlap with inputs or each other. S, X, T > 0, sigma > 0 (not checked
  * per element: a non-positive element yields NaN/inf in its own outputs only).
  * N() uses the Abramowitz-Stegun 26.2.17 approximation (|err| < 7.5e-8).
- * Launch override: grid_ctas, block_threads honoured.
+ * Launch override: grid_ctas honoured.
  * =========================================================================== */
 lime_status lime_map_blackscholes(const float *S, const float *X, const float *T, int64_t n,
                                   float r, float sigma, float *call, float *put, void *stream);
 
 /* Fused map+reduce (`!` over `@` without materialising the map, L160-163,
  * L188-189; R6): sums[0] = sum_i call[i], sums[1] = sum_i put[i]
- * (device double[2]), accumulated in fp64 from the CTA level up, CTA partials
- * combined in fixed index order by the last CTA (deterministic for a given
- * launch configuration). ws: lime_reduce_workspace_bytes() bytes. */
+ * (device double[2]), accumulated in fp64 from the warp level up (per-thread
+ * partials fp32), CTA partials combined in fixed index order by the last CTA
+ * (deterministic for a given launch configuration). The element is the same
+ * closed form rearranged for summation: with A = S N(d1) - S/2 and
+ * B = K N(d2) - K/2 (K = X e^{-rT}), call = (A - B) + (S - K)/2 and
+ * put = (A - B) - (S - K)/2, so only the sums of A - B and S - K are formed
+ * (put-call parity holds by construction). Tolerance vs the
+ * oracle: 1e-5 relative on each sum. ws: lime_reduce_workspace_bytes() bytes.
+ * Launch override: grid_ctas honoured. */
 lime_status lime_map_reduce_blackscholes_sum(const float *S, const float *X, const float *T,
                                              int64_t n, float r, float sigma, double *sums,
                                              void *ws, size_t ws_bytes, void *stream);
@@ -208,7 +219,8 @@ lime_status lime_map_reduce_blackscholes_sum(const float *S, const float *X, con
  * cyclic multi-GPU shard). width, height > 0; 0 <= row_first < height;
  * row_stride >= 1; every addressed py < height; max_iter >= 0.
  * ws: lime_mandelbrot_workspace_bytes() bytes (tile-queue counters).
- * Launch override: grid_ctas honoured.
+ * Launch override: grid_ctas honoured; per_thread 1..8 selects the warp tile
+ * shape / vote interval (tools/tune_mandel.py; results bit-identical).
  * =========================================================================== */
 size_t lime_mandelbrot_workspace_bytes(void);
 lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first,
@@ -222,7 +234,13 @@ lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first
  * A [M][K] bf16 bits (uint16), Bt [N][K] bf16 bits (K-major both), C [M][N]
  * float (fp32 accumulate, tcgen05 tensor cores). M, N >= 1; K >= 8 and
  * K % 8 == 0 (16-byte TMA row stride); A, Bt, C 16-B aligned; C must not
- * overlap A or Bt.
+ * overlap A or Bt. Accumulation order is fixed by K (per-K-slice MMAs in
+ * order), so C does not depend on the launch configuration. For M >= 256 a
+ * CTA pair (cta_group::2) computes 256 x 256 tiles; C is written by TMA tensor
+ * stores when N % 4 == 0, else by direct stores (same bits).
+ * Launch override: grid_ctas (persistent CTAs); block_threads = tile raster
+ * group; per_thread 1 = one-CTA kernel, 2 = pair kernel, 3 = pair kernel with
+ * the direct-store epilogue.
  * =========================================================================== */
 lime_status lime_map_matmul_bf16(const uint16_t *A, const uint16_t *Bt, float *C, int64_t M,
                                  int64_t N, int64_t K, void *stream);
