@@ -482,6 +482,27 @@ def run_extras(peaks, flush):
         del bd
     del acc1m
 
+    # config-5 strong scaling on ONE GPU, compute only: the force map of the rank-0 shard at P = 1, 2, 4,
+    # 8 (2^20/P targets x 2^20 sources, the launch each rank runs); E(P) = T_1 / (P T_P). The per-step
+    # all-gather (2^20/P x 16 B out, 16 MiB in per rank) is what the driver's N-GPU runs add on top.
+    bd = torch.from_numpy(b1m).cuda()
+    acc_full = torch.empty((1 << 20, 4), dtype=torch.float32, device="cuda")
+    shard_ms = {}
+    for P in (1, 2, 4, 8):
+        cnt = (1 << 20) // P
+        shard_ms[P], _ = time_launches(lambda: lime.map_nbody(bd, EPS2, 0, cnt, out=acc_full[:cnt]), 3, 1, flush)
+    out["nbody_1m_shard_scaling_probe"] = {
+        "workload": "config-5 force map of one rank's shard at P = 1, 2, 4, 8 on one GPU (compute only)",
+        "ms_per_launch": {str(P): v for P, v in shard_ms.items()},
+        "compute_strong_scaling_efficiency": {str(P): shard_ms[1] / (P * v) for P, v in shard_ms.items()},
+        "value": float(1 << 17) * (1 << 20) / (shard_ms[8] * 1e-3), "unit": "interactions/s (one P = 8 shard)",
+        "projected_8gpu_interactions_per_s_compute_only": float(1 << 20) * (1 << 20) / (shard_ms[8] * 1e-3),
+        "roofline": {"bound": "alu", "achieved": FLOP_PER_INTERACTION * float(1 << 17) * (1 << 20) / (shard_ms[8] * 1e-3) / 1e12,
+                     "peak": fp32, "unit": "TFLOP/s",
+                     "frac": FLOP_PER_INTERACTION * float(1 << 17) * (1 << 20) / (shard_ms[8] * 1e-3) / 1e12 / fp32,
+                     "traffic": None}}
+    del bd, acc_full
+
     # F3: double-precision N-Body (Table 3) at the config-5 per-GPU shape of P = 8; FP64-pipe
     # bound: 16 FP64 ops per interaction at 64 lanes/clk/SM (microbench: 58.9 measured)
     b64 = torch.from_numpy(inputs.nbody_bodies(1 << 20, seed=5).astype(np.float64)).cuda()
