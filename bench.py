@@ -478,7 +478,7 @@ def run_extras(peaks, flush):
                     "fp32_lane_ops_per_interaction": ops,
                     "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s", "frac": ach / fp32,
                                  "fp32_pipe_frac": ops * inter / (med * 1e-3) / (SMS_B200 * 128 * SM_MAX_MHZ_NOMINAL * 1e6),
-                                 "traffic": None}}
+                                 "traffic": ncu_traffic("nbody_force_1m_p8") if ops == FP32_LANE_OPS_UNIFORM_MASS else None}}
         del bd
     del acc1m
 

@@ -34,7 +34,11 @@ def main(tag):
     tp = os.path.join(prof, "ncu_traffic.json")
     old = json.load(open(tp)) if os.path.exists(tp) else {}
     old.update(traffic)
-    old["_source"] = f"dram__bytes_read.sum + dram__bytes_write.sum per launch, ncu --set full, round {tag}"
+    rounds = old.get("_rounds", {})
+    rounds.update({k: tag for k in traffic})
+    old["_rounds"] = rounds
+    old["_source"] = ("dram__bytes_read.sum + dram__bytes_write.sum per launch, ncu --set full; "
+                      "latest round that profiled each kernel in _rounds")
     with open(tp, "w") as f:
         json.dump(old, f, indent=1)
     for fn in (f"launches_{tag}.csv", f"bench_{tag}.json"):
