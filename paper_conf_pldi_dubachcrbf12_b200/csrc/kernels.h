@@ -25,8 +25,14 @@ namespace nbody {
 // ones 256-body chunks and up to 16 splits.
 constexpr int kChunk = 256;
 constexpr int kMaxSplits = 16;
-constexpr int kChunkSmall = 128;
-constexpr int kMaxSplitsSmall = 32;
+#ifndef LIME_CHUNK_SMALL            // compile-time A/B overrides (tools/); the defaults are the product
+#define LIME_CHUNK_SMALL 128
+#endif
+#ifndef LIME_MAX_SPLITS_SMALL
+#define LIME_MAX_SPLITS_SMALL 32
+#endif
+constexpr int kChunkSmall = LIME_CHUNK_SMALL;
+constexpr int kMaxSplitsSmall = LIME_MAX_SPLITS_SMALL;
 constexpr int64_t kSmallMaxSources = 8192;
 int chunk_len(int64_t n_src);
 int64_t chunks_per_split(int64_t n_src);
