@@ -27,6 +27,14 @@
 namespace lime {
 namespace nbody {
 
+#ifndef LIME_UNIT_UNROLL           // compile-time A/B overrides (tools/ab_nbody_1m.py); defaults are the product
+#define LIME_UNIT_UNROLL 8            // r01t A/B: 8 beats 2, 4, 16 (profiles/experiments/nbody_unroll_ab_r01*.jsonl)
+#endif
+#ifndef LIME_BODY_UNROLL
+#define LIME_BODY_UNROLL 4
+#endif
+constexpr int kUnitUnroll = LIME_UNIT_UNROLL;
+constexpr int kBodyUnroll = LIME_BODY_UNROLL;
 constexpr int kTileJ = 1024;   // sources per shared-memory stage (16 KB)
 static_assert(kTileJ % kChunk == 0 && kTileJ % kChunkSmall == 0, "stage must hold whole chunks");
 
@@ -381,7 +389,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constan
             it.chunk_begin();
             if constexpr (UNIT) {
                 if (c1 - c0 == CHUNK) {
-#pragma unroll 4
+#pragma unroll kUnitUnroll
                     for (int j = c0; j < c0 + CHUNK; ++j) it.body_unit(sb[j], eps2);
                 } else {
                     for (int j = c0; j < c1; ++j) it.body_unit(sb[j], eps2);
@@ -389,7 +397,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constan
                 it.chunk_end_scaled(sb[c0].w);
             } else {
                 if (c1 - c0 == CHUNK) {
-#pragma unroll 4
+#pragma unroll kBodyUnroll
                     for (int j = c0; j < c0 + CHUNK; ++j) it.body(sb[j], eps2);
                 } else {
                     for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
