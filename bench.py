@@ -300,9 +300,6 @@ def run_nbody(args, rank, world, local):
                 "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 flop x 1965 MHz (microbench: 124.9-127.9 lane-ops/clk/SM)",
                 "flop_per_interaction": FLOP_PER_INTERACTION,
                 "fp32_lane_ops_per_interaction": lane_ops,
-                "element_form": "mass factored out of each chunk sum (equal masses, DESIGN.md R11)" if uniform_mass
-                                else "per-body mass multiply",
-                "fp32_lane_ops_per_interaction": lane_ops,
                 "element_form": ("mass factored out of each chunk sum (equal masses, DESIGN.md R11)" if uniform_mass
                                  else "per-body mass multiply"),
                 "fp32_pipe_frac_at_observed_clock": pipe_frac, "observed_sm_mhz": obs_mhz,

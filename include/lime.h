@@ -233,7 +233,9 @@ lime_status lime_map_mandelbrot(int32_t width, int32_t height, int32_t row_first
  * in the paper; R8): C[i][j] = sum_k A[i][k] * Bt[j][k].
  * A [M][K] bf16 bits (uint16), Bt [N][K] bf16 bits (K-major both), C [M][N]
  * float (fp32 accumulate, tcgen05 tensor cores). M, N >= 1; K >= 8 and
- * K % 8 == 0 (16-byte TMA row stride); A, Bt, C 16-B aligned; C must not
+ * K % 8 == 0 (16-byte TMA row stride); M, N, K <= 2^31 - 512 and
+ * ceil(M/256) * ceil(N/256) <= 2^31 - 1 (int32 rows, TMA coordinates and tile
+ * indices; else LIME_ERR_INVALID_ARG); A, Bt, C 16-B aligned; C must not
  * overlap A or Bt. Accumulation order is fixed by K (per-K-slice MMAs in
  * order), so C does not depend on the launch configuration. For M >= 256 a
  * CTA pair (cta_group::2) computes 256 x 256 tiles; C is written by TMA tensor

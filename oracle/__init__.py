@@ -192,14 +192,29 @@ def mandelbrot(width, height, row_first, row_stride, row_count, x0, y0, dx, dy, 
     threads (each call is the single-threaded C loop on a disjoint row range)."""
     out = np.zeros((row_count, width), dtype=np.int32)
     L = lib()
+    threads = max(1, min(threads, row_count if row_count > 0 else 1))
+    if threads == 1:
+        if row_count > 0:
+            L.oracle_mandelbrot(width, height, row_first, row_stride, row_count, float(x0), float(y0),
+                                float(dx), float(dy), max_iter, out.ctypes.data)
+        return out
 
-    def work(lo, hi):
-        if hi > lo:
-            L.oracle_mandelbrot(width, height, row_first + lo * row_stride, row_stride, hi - lo,
-                                float(x0), float(y0), float(dx), float(dy), max_iter,
-                                out[lo:hi].ctypes.data)
+    # Thread k takes rows k, k + threads, ... (the escape time varies strongly from row to row, so
+    # interleaving balances the threads); each part is the same single-threaded C loop over a
+    # row set with stride row_stride * threads, written into its own dense array.
+    def work(k):
+        cnt = len(range(k, row_count, threads))
+        if cnt:
+            part = np.zeros((cnt, width), dtype=np.int32)
+            L.oracle_mandelbrot(width, height, row_first + k * row_stride, row_stride * threads, cnt,
+                                float(x0), float(y0), float(dx), float(dy), max_iter, part.ctypes.data)
+            out[k::threads] = part
 
-    _parallel(work, row_count, threads, chunked=True)
+    ts = [threading.Thread(target=work, args=(k,)) for k in range(threads)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
     return out
 
 

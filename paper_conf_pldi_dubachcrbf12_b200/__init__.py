@@ -105,7 +105,12 @@ def _stream(device) -> int:
     return torch.cuda.current_stream(device).cuda_stream
 
 
-def _dev_tensor(t: torch.Tensor, dtype, name: str, ndim_last: int | None = None):
+def _dev_tensor(t: torch.Tensor, dtype, name: str, ndim_last: int | None = None, numel: int | None = None,
+                device=None):
+    """Validate one operand or output: a contiguous CUDA tensor of `dtype`, optionally of shape
+    [n][ndim_last], with exactly `numel` elements, on `device`. The C ABI cannot see tensor extents,
+    so every size the kernels rely on is checked here (a mistake would otherwise be an out-of-bounds
+    device access, not an error)."""
     if not isinstance(t, torch.Tensor) or not t.is_cuda:
         raise TypeError(f"{name} must be a CUDA tensor")
     if t.dtype != dtype:
@@ -114,7 +119,18 @@ def _dev_tensor(t: torch.Tensor, dtype, name: str, ndim_last: int | None = None)
         raise ValueError(f"{name} must be contiguous")
     if ndim_last is not None and (t.dim() != 2 or t.shape[1] != ndim_last):
         raise ValueError(f"{name} must have shape [n][{ndim_last}]")
+    if numel is not None and t.numel() != numel:
+        raise ValueError(f"{name} must have {numel} elements, got {t.numel()}")
+    if device is not None and t.device != torch.device(device):
+        raise ValueError(f"{name} is on {t.device}, expected {device} (all operands on one device)")
     return t
+
+
+def _device(device) -> torch.device:
+    dev = torch.device(device)
+    if dev.type != "cuda":
+        raise TypeError(f"device must be a CUDA device, got {dev}")
+    return torch.device("cuda", dev.index if dev.index is not None else torch.cuda.current_device())
 
 
 # Zero-filled, self-resetting workspaces, one per (device, stream, kind).
@@ -166,21 +182,28 @@ def nbody_splits(n_src: int) -> int:
     return int(load().lime_nbody_splits(n_src))
 
 
+def _target_range(n: int, tgt_begin: int, tgt_count: int | None) -> int:
+    """Element count of the output range (the C ABI itself rejects a range outside [0, n))."""
+    if tgt_count is None:
+        tgt_count = n - tgt_begin
+    return max(int(tgt_count), 0)
+
+
 def map_nbody(bodies: torch.Tensor, eps2: float, tgt_begin: int = 0, tgt_count: int | None = None,
               out: torch.Tensor | None = None) -> torch.Tensor:
     """accel[t] for targets [tgt_begin, tgt_begin+tgt_count) of bodies [n][4] (x,y,z,m)."""
     L = load()
     _dev_tensor(bodies, torch.float32, "bodies", 4)
     n = bodies.shape[0]
-    if tgt_count is None:
-        tgt_count = n - tgt_begin
+    tgt_count = _target_range(n, tgt_begin, tgt_count)
+    dev = bodies.device
     if out is None:
-        out = torch.empty((max(tgt_count, 0), 4), dtype=torch.float32, device=bodies.device)
-    _dev_tensor(out, torch.float32, "out", 4)
-    nbytes = L.lime_map_nbody_workspace_bytes(n, max(tgt_count, 0))
-    ws = workspace(bodies.device, "nbody", nbytes)
-    _check(L.lime_map_nbody(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
-                            ws.data_ptr(), ws.numel(), _stream(bodies.device)), "lime_map_nbody")
+        out = torch.empty((tgt_count, 4), dtype=torch.float32, device=dev)
+    _dev_tensor(out, torch.float32, "out", 4, numel=4 * tgt_count, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "nbody", L.lime_map_nbody_workspace_bytes(n, tgt_count))
+        _check(L.lime_map_nbody(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
+                                ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_nbody")
     return out
 
 
@@ -190,24 +213,28 @@ def map_nbody_f64(bodies: torch.Tensor, eps2: float, tgt_begin: int = 0, tgt_cou
     L = load()
     _dev_tensor(bodies, torch.float64, "bodies", 4)
     n = bodies.shape[0]
-    if tgt_count is None:
-        tgt_count = n - tgt_begin
+    tgt_count = _target_range(n, tgt_begin, tgt_count)
+    dev = bodies.device
     if out is None:
-        out = torch.empty((max(tgt_count, 0), 4), dtype=torch.float64, device=bodies.device)
-    _dev_tensor(out, torch.float64, "out", 4)
-    ws = workspace(bodies.device, "nbody64", L.lime_map_nbody_f64_workspace_bytes(n, max(tgt_count, 0)))
-    _check(L.lime_map_nbody_f64(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
-                                ws.data_ptr(), ws.numel(), _stream(bodies.device)), "lime_map_nbody_f64")
+        out = torch.empty((tgt_count, 4), dtype=torch.float64, device=dev)
+    _dev_tensor(out, torch.float64, "out", 4, numel=4 * tgt_count, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "nbody64", L.lime_map_nbody_f64_workspace_bytes(n, tgt_count))
+        _check(L.lime_map_nbody_f64(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, out.data_ptr(),
+                                    ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_nbody_f64")
     return out
 
 
 def map_nbody_integrate(pos: torch.Tensor, vel: torch.Tensor, accel: torch.Tensor, dt: float) -> None:
     """In-place semi-implicit Euler step of pos/vel ([n][4] each)."""
     L = load()
-    for t, nm in ((pos, "pos"), (vel, "vel"), (accel, "accel")):
-        _dev_tensor(t, torch.float32, nm, 4)
-    _check(L.lime_map_nbody_integrate(pos.data_ptr(), vel.data_ptr(), accel.data_ptr(), pos.shape[0], dt,
-                                      _stream(pos.device)), "lime_map_nbody_integrate")
+    _dev_tensor(pos, torch.float32, "pos", 4)
+    n, dev = pos.shape[0], pos.device
+    _dev_tensor(vel, torch.float32, "vel", 4, numel=4 * n, device=dev)
+    _dev_tensor(accel, torch.float32, "accel", 4, numel=4 * n, device=dev)
+    with torch.cuda.device(dev):
+        _check(L.lime_map_nbody_integrate(pos.data_ptr(), vel.data_ptr(), accel.data_ptr(), n, dt, _stream(dev)),
+               "lime_map_nbody_integrate")
 
 
 def nbody_simulate(pos: torch.Tensor, vel: torch.Tensor, steps: int, eps2: float, dt: float) -> None:
@@ -215,13 +242,12 @@ def nbody_simulate(pos: torch.Tensor, vel: torch.Tensor, steps: int, eps2: float
     persistent launch for n <= 8192."""
     L = load()
     _dev_tensor(pos, torch.float32, "pos", 4)
-    _dev_tensor(vel, torch.float32, "vel", 4)
-    if vel.shape[0] != pos.shape[0] or vel.device != pos.device:
-        raise ValueError("pos and vel must have the same length and device")
-    n = pos.shape[0]
-    ws = workspace(pos.device, "nbody_sim", L.lime_nbody_simulate_workspace_bytes(n))
-    _check(L.lime_nbody_simulate(pos.data_ptr(), vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(), ws.numel(),
-                                 _stream(pos.device)), "lime_nbody_simulate")
+    n, dev = pos.shape[0], pos.device
+    _dev_tensor(vel, torch.float32, "vel", 4, numel=4 * n, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "nbody_sim", L.lime_nbody_simulate_workspace_bytes(n))
+        _check(L.lime_nbody_simulate(pos.data_ptr(), vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(), ws.numel(),
+                                     _stream(dev)), "lime_nbody_simulate")
 
 
 def nbody_simulate_host(h_pos: torch.Tensor, h_vel: torch.Tensor, steps: int, eps2: float, dt: float,
@@ -231,36 +257,49 @@ def nbody_simulate_host(h_pos: torch.Tensor, h_vel: torch.Tensor, steps: int, ep
     for t, nm in ((h_pos, "h_pos"), (h_vel, "h_vel")):
         if t.is_cuda or t.dtype != torch.float32 or not t.is_contiguous() or t.dim() != 2 or t.shape[1] != 4:
             raise ValueError(f"{nm} must be a contiguous host float32 [n][4] tensor")
+    if h_vel.shape[0] != h_pos.shape[0]:
+        raise ValueError("h_pos and h_vel must have the same length")
     n = h_pos.shape[0]
-    dev = torch.device(device)
-    ws = workspace(dev, "nbody_host", L.lime_nbody_simulate_host_workspace_bytes(n))
-    _check(L.lime_nbody_simulate_host(h_pos.data_ptr(), h_vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(),
-                                      ws.numel(), _stream(dev)), "lime_nbody_simulate_host")
+    dev = _device(device)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "nbody_host", L.lime_nbody_simulate_host_workspace_bytes(n))
+        _check(L.lime_nbody_simulate_host(h_pos.data_ptr(), h_vel.data_ptr(), n, steps, eps2, dt, ws.data_ptr(),
+                                          ws.numel(), _stream(dev)), "lime_nbody_simulate_host")
 
 
 # ------------------------------------------------------------------ Black-Scholes
+def _options(S, X, T):
+    _dev_tensor(S, torch.float32, "S")
+    n, dev = S.numel(), S.device
+    _dev_tensor(X, torch.float32, "X", numel=n, device=dev)
+    _dev_tensor(T, torch.float32, "T", numel=n, device=dev)
+    return n, dev
+
+
 def map_blackscholes(S, X, T, r: float, sigma: float, call=None, put=None):
     L = load()
-    for t, nm in ((S, "S"), (X, "X"), (T, "T")):
-        _dev_tensor(t, torch.float32, nm)
-    n = S.numel()
-    call = torch.empty(n, dtype=torch.float32, device=S.device) if call is None else call
-    put = torch.empty(n, dtype=torch.float32, device=S.device) if put is None else put
-    _check(L.lime_map_blackscholes(S.data_ptr(), X.data_ptr(), T.data_ptr(), n, r, sigma, call.data_ptr(),
-                                   put.data_ptr(), _stream(S.device)), "lime_map_blackscholes")
+    n, dev = _options(S, X, T)
+    call = torch.empty(n, dtype=torch.float32, device=dev) if call is None else call
+    put = torch.empty(n, dtype=torch.float32, device=dev) if put is None else put
+    _dev_tensor(call, torch.float32, "call", numel=n, device=dev)
+    _dev_tensor(put, torch.float32, "put", numel=n, device=dev)
+    with torch.cuda.device(dev):
+        _check(L.lime_map_blackscholes(S.data_ptr(), X.data_ptr(), T.data_ptr(), n, r, sigma, call.data_ptr(),
+                                       put.data_ptr(), _stream(dev)), "lime_map_blackscholes")
     return call, put
 
 
 def map_reduce_blackscholes_sum(S, X, T, r: float, sigma: float, out=None) -> torch.Tensor:
     """Device float64[2] = (sum call, sum put), fused (the map is never materialised)."""
     L = load()
-    for t, nm in ((S, "S"), (X, "X"), (T, "T")):
-        _dev_tensor(t, torch.float32, nm)
-    out = torch.empty(2, dtype=torch.float64, device=S.device) if out is None else out
-    ws = workspace(S.device, "reduce", L.lime_reduce_workspace_bytes())
-    _check(L.lime_map_reduce_blackscholes_sum(S.data_ptr(), X.data_ptr(), T.data_ptr(), S.numel(), r, sigma,
-                                              out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(S.device)),
-           "lime_map_reduce_blackscholes_sum")
+    n, dev = _options(S, X, T)
+    out = torch.empty(2, dtype=torch.float64, device=dev) if out is None else out
+    _dev_tensor(out, torch.float64, "out", numel=2, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "reduce", L.lime_reduce_workspace_bytes())
+        _check(L.lime_map_reduce_blackscholes_sum(S.data_ptr(), X.data_ptr(), T.data_ptr(), n, r, sigma,
+                                                  out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)),
+               "lime_map_reduce_blackscholes_sum")
     return out
 
 
@@ -271,11 +310,13 @@ def map_mandelbrot(width: int, height: int, x0: float, y0: float, dx: float, dy:
     L = load()
     if row_count is None:
         row_count = len(range(row_first, height, row_stride))
-    dev = torch.device(device)
+    dev = out.device if out is not None else _device(device)
     out = torch.empty((row_count, width), dtype=torch.int32, device=dev) if out is None else out
-    ws = workspace(dev, "mandel", L.lime_mandelbrot_workspace_bytes())
-    _check(L.lime_map_mandelbrot(width, height, row_first, row_stride, row_count, x0, y0, dx, dy, max_iter,
-                                 out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_mandelbrot")
+    _dev_tensor(out, torch.int32, "out", numel=max(row_count, 0) * max(width, 0), device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "mandel", L.lime_mandelbrot_workspace_bytes())
+        _check(L.lime_map_mandelbrot(width, height, row_first, row_stride, row_count, x0, y0, dx, dy, max_iter,
+                                     out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_mandelbrot")
     return out
 
 
@@ -284,14 +325,19 @@ def map_matmul_bf16(A: torch.Tensor, Bt: torch.Tensor, out=None) -> torch.Tensor
     """C[M][N] fp32 = A[M][K] . Bt[N][K]^T (bf16 in, tcgen05 tensor cores)."""
     L = load()
     _dev_tensor(A, torch.bfloat16, "A")
-    _dev_tensor(Bt, torch.bfloat16, "Bt")
+    if A.dim() != 2:
+        raise ValueError("A must be [M][K]")
     M, K = A.shape
+    dev = A.device
+    _dev_tensor(Bt, torch.bfloat16, "Bt", device=dev)
+    if Bt.dim() != 2 or Bt.shape[1] != K:
+        raise ValueError("Bt must be [N][K] with A's K")
     N = Bt.shape[0]
-    if Bt.shape[1] != K:
-        raise ValueError("A and Bt must share K")
-    out = torch.empty((M, N), dtype=torch.float32, device=A.device) if out is None else out
-    _check(L.lime_map_matmul_bf16(A.data_ptr(), Bt.data_ptr(), out.data_ptr(), M, N, K, _stream(A.device)),
-           "lime_map_matmul_bf16")
+    out = torch.empty((M, N), dtype=torch.float32, device=dev) if out is None else out
+    _dev_tensor(out, torch.float32, "out", numel=M * N, device=dev)
+    with torch.cuda.device(dev):
+        _check(L.lime_map_matmul_bf16(A.data_ptr(), Bt.data_ptr(), out.data_ptr(), M, N, K, _stream(dev)),
+               "lime_map_matmul_bf16")
     return out
 
 
@@ -301,12 +347,14 @@ def map_coulomb(atoms: torch.Tensor, nx: int, ny: int, z: float, h: float, p_beg
     """Coulombic potential V[p] over lattice points [p_begin, p_begin+p_count) of an nx x ny slice."""
     L = load()
     _dev_tensor(atoms, torch.float32, "atoms", 4)
-    if p_count is None:
-        p_count = nx * ny - p_begin
-    out = torch.empty(max(p_count, 0), dtype=torch.float32, device=atoms.device) if out is None else out
-    ws = workspace(atoms.device, "coulomb", L.lime_map_coulomb_workspace_bytes(atoms.shape[0], max(p_count, 0)))
-    _check(L.lime_map_coulomb(atoms.data_ptr(), atoms.shape[0], nx, ny, p_begin, p_count, z, h, out.data_ptr(),
-                              ws.data_ptr(), ws.numel(), _stream(atoms.device)), "lime_map_coulomb")
+    dev = atoms.device
+    p_count = _target_range(nx * ny, p_begin, p_count)
+    out = torch.empty(p_count, dtype=torch.float32, device=dev) if out is None else out
+    _dev_tensor(out, torch.float32, "out", numel=p_count, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "coulomb", L.lime_map_coulomb_workspace_bytes(atoms.shape[0], p_count))
+        _check(L.lime_map_coulomb(atoms.data_ptr(), atoms.shape[0], nx, ny, p_begin, p_count, z, h, out.data_ptr(),
+                                  ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_coulomb")
     return out
 
 
@@ -314,15 +362,17 @@ def map_mriq(kspace: torch.Tensor, voxels: torch.Tensor, x_begin: int = 0, x_cou
              out=None) -> torch.Tensor:
     """MRI-Q: (Qr, Qi) [x_count][2] for voxels [x_begin, x_begin+x_count)."""
     L = load()
-    _dev_tensor(kspace, torch.float32, "kspace", 5)
     _dev_tensor(voxels, torch.float32, "voxels", 3)
+    dev = voxels.device
+    _dev_tensor(kspace, torch.float32, "kspace", 5, device=dev)
     n_x = voxels.shape[0]
-    if x_count is None:
-        x_count = n_x - x_begin
-    out = torch.empty((max(x_count, 0), 2), dtype=torch.float32, device=voxels.device) if out is None else out
-    ws = workspace(voxels.device, "mriq", L.lime_map_mriq_workspace_bytes(kspace.shape[0], max(x_count, 0)))
-    _check(L.lime_map_mriq(kspace.data_ptr(), kspace.shape[0], voxels.data_ptr(), n_x, x_begin, x_count,
-                           out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(voxels.device)), "lime_map_mriq")
+    x_count = _target_range(n_x, x_begin, x_count)
+    out = torch.empty((x_count, 2), dtype=torch.float32, device=dev) if out is None else out
+    _dev_tensor(out, torch.float32, "out", numel=2 * x_count, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "mriq", L.lime_map_mriq_workspace_bytes(kspace.shape[0], x_count))
+        _check(L.lime_map_mriq(kspace.data_ptr(), kspace.shape[0], voxels.data_ptr(), n_x, x_begin, x_count,
+                               out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_mriq")
     return out
 
 
@@ -330,11 +380,15 @@ def map_mriq(kspace: torch.Tensor, voxels: torch.Tensor, x_begin: int = 0, x_cou
 def map_series(n0: int, count: int, dtype=torch.float32, device="cuda", out=None) -> torch.Tensor:
     """JG-Series coefficient pairs (a_n, b_n) for n in [n0, n0+count) -> [count][2]."""
     L = load()
-    dev = torch.device(device)
+    if dtype not in (torch.float32, torch.float64):
+        raise TypeError("dtype must be float32 or float64")
+    dev = out.device if out is not None else _device(device)
     out = torch.empty((count, 2), dtype=dtype, device=dev) if out is None else out
-    ws = workspace(dev, "series", L.lime_map_series_workspace_bytes())
+    _dev_tensor(out, dtype, "out", numel=2 * max(count, 0), device=dev)
     fn = L.lime_map_series_f64 if dtype == torch.float64 else L.lime_map_series_f32
-    _check(fn(n0, count, out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_series")
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "series", L.lime_map_series_workspace_bytes())
+        _check(fn(n0, count, out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_series")
     return out
 
 
@@ -355,10 +409,15 @@ def map_idea(data: torch.Tensor, subkeys, out=None) -> torch.Tensor:
     import numpy as np
     L = load()
     _dev_tensor(data, torch.uint8, "data")
+    dev = data.device
     z = np.ascontiguousarray(subkeys, dtype=np.uint16)
+    if z.shape != (52,):
+        raise ValueError("subkeys must be 52 16-bit words")
     out = torch.empty_like(data) if out is None else out
-    _check(L.lime_map_idea(data.data_ptr(), out.data_ptr(), data.numel(), z.ctypes.data, _stream(data.device)),
-           "lime_map_idea")
+    _dev_tensor(out, torch.uint8, "out", numel=data.numel(), device=dev)
+    with torch.cuda.device(dev):
+        _check(L.lime_map_idea(data.data_ptr(), out.data_ptr(), data.numel(), z.ctypes.data, _stream(dev)),
+               "lime_map_idea")
     return out
 
 
@@ -371,11 +430,14 @@ def _reduce(op: str, x: torch.Tensor, out=None) -> torch.Tensor:
     if x.dtype not in _RED_DT:
         raise TypeError(f"unsupported dtype {x.dtype}")
     _dev_tensor(x, x.dtype, "x")
-    out = torch.empty((), dtype=x.dtype, device=x.device) if out is None else out
-    ws = workspace(x.device, "reduce", L.lime_reduce_workspace_bytes())
+    dev = x.device
+    out = torch.empty((), dtype=x.dtype, device=dev) if out is None else out
+    _dev_tensor(out, x.dtype, "out", numel=1, device=dev)
     fn = getattr(L, f"lime_reduce_{op}_{_RED_DT[x.dtype]}")
-    _check(fn(x.data_ptr(), x.numel(), out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(x.device)),
-           f"lime_reduce_{op}")
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "reduce", L.lime_reduce_workspace_bytes())
+        _check(fn(x.data_ptr(), x.numel(), out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)),
+               f"lime_reduce_{op}")
     return out
 
 

@@ -8,6 +8,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 #include "../../include/lime.h"
 #include "common.cuh"
@@ -26,8 +30,40 @@ bool pdl_enabled() {
     return on;
 }
 
+cudaError_t ensure_dynamic_smem(const void* kernel, int bytes) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    static std::mutex mu;
+    static std::map<std::pair<const void*, int>, int> set;     // (kernel, device) -> bytes allowed
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = set.find({kernel, dev});
+    if (it != set.end() && it->second >= bytes) return cudaSuccess;
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess) set[{kernel, dev}] = bytes;
+    return e;
+}
+
+int cached_occupancy(const void* kernel, int block, size_t smem) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return 0; }
+    static std::mutex mu;
+    static std::map<std::tuple<const void*, int, size_t, int>, int> occ;
+    std::lock_guard<std::mutex> lock(mu);
+    const auto key = std::make_tuple(kernel, block, smem, dev);
+    auto it = occ.find(key);
+    if (it != occ.end()) return it->second;
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, block, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    occ[key] = b;
+    return b;
+}
+
 int device_num_sms() {
-    static int cached[64] = {0};
+    static std::atomic<int> cached[64];   // zero-initialised (static storage)
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return kNumSMsB200;
     if (cached[dev] == 0) {
@@ -57,7 +93,7 @@ static bool overlap(const void* a, size_t abytes, const void* b, size_t bbytes) 
 }
 
 static lime_status check_device() {
-    static int ok_cache[64] = {0};   // 0 unknown, 1 ok, 2 bad
+    static std::atomic<int> ok_cache[64];   // 0 unknown, 1 ok, 2 bad
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) {
@@ -449,8 +485,12 @@ lime_status lime_map_matmul_bf16(const uint16_t* A, const uint16_t* Bt, float* C
                                  void* stream) {
     if (M < 1 || N < 1 || K < 8 || (K % 8) != 0)
         return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: need M, N >= 1 and K >= 8, K %% 8 == 0");
-    if (M > (1LL << 31) || N > (1LL << 31) || K > (1LL << 31))
-        return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: dimension exceeds 2^31");
+    // the kernels index rows, TMA coordinates and tiles in int32: every padded dimension and the
+    // tile count must stay below 2^31
+    constexpr int64_t kDimMax = (1LL << 31) - 512;
+    if (M > kDimMax || N > kDimMax || K > kDimMax ||
+        ((M + 255) / 256) * ((N + 255) / 256) > static_cast<int64_t>(INT32_MAX))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: dimension or tile count exceeds the int32 range");
     if (!A || !Bt || !C) return fail(LIME_ERR_INVALID_ARG, "lime_map_matmul_bf16: null pointer");
     if (!aligned16(A) || !aligned16(Bt) || !aligned16(C))
         return fail(LIME_ERR_MISALIGNED, "lime_map_matmul_bf16: A, Bt, C must be 16-byte aligned");

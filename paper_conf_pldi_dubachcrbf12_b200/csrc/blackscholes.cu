@@ -282,15 +282,9 @@ static Consts make_consts(float r, float sigma) {
 static int grid_for(const void* kernel, int64_t n) {
     const int ov = launch_override().grid_ctas;
     if (ov > 0) return ov;
-    static int per_sm[2] = {0, 0};
-    const int idx = (kernel == reinterpret_cast<const void*>(&map_kernel)) ? 0 : 1;
-    if (per_sm[idx] == 0) {
-        int b = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, 256, 0);
-        per_sm[idx] = b > 0 ? b : 1;
-    }
+    const int per_sm = mx(1, cached_occupancy(kernel, 256, 0));
     const int64_t need = ceil_div<int64_t>(mx<int64_t>(n >> 2, 1), 256);
-    return static_cast<int>(mn<int64_t>(need, static_cast<int64_t>(per_sm[idx]) * device_num_sms()));
+    return static_cast<int>(mn<int64_t>(need, static_cast<int64_t>(per_sm) * device_num_sms()));
 }
 
 cudaError_t launch_map(const float* S, const float* X, const float* T, int64_t n, float r, float sigma,

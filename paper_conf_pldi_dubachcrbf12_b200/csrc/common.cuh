@@ -184,6 +184,12 @@ __device__ __forceinline__ void pdl_enter() {
     asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 bool pdl_enabled();   // false when LIME_NO_PDL is set in the environment (A/B and debugging)
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device): the attribute is
+// per device, so the cache is keyed by the current device; thread-safe (abi.cu).
+cudaError_t ensure_dynamic_smem(const void* kernel, int bytes);
+// Occupancy (resident CTAs per SM) of `kernel` at `block` threads and `smem` dynamic bytes, cached
+// per (kernel, block, smem, device); thread-safe (abi.cu). Returns >= 1, or 0 on error.
+int cached_occupancy(const void* kernel, int block, size_t smem);
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t stream,
                               Args... args) {

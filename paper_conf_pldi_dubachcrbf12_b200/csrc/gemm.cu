@@ -540,13 +540,8 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
         std::memset(&mc, 0, sizeof mc);
         p.tma_store = ((N & 3) == 0 && (reinterpret_cast<uintptr_t>(C) & 15) == 0 && ov.per_thread != 3 &&
                        make_map_c(&mc, C, M, N)) ? 1 : 0;
-        static bool attr2 = false;
-        if (!attr2) {
-            cudaError_t e = cudaFuncSetAttribute(gemm2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                 static_cast<int>(two::kSmemBytes));
-            if (e != cudaSuccess) return e;
-            attr2 = true;
-        }
+        cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&gemm2_kernel), static_cast<int>(two::kSmemBytes));
+        if (e != cudaSuccess) return e;
         int clusters = ov.grid_ctas > 0 ? mx(1, ov.grid_ctas / 2) : device_num_sms() / 2;
         clusters = mn(clusters, p.num_tiles);
         gemm2_kernel<<<2 * clusters, kThreads, two::kSmemBytes, stream>>>(ma, mb, mc, p);
@@ -562,13 +557,8 @@ cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t
     p.num_n = static_cast<int>(ceil_div<int64_t>(N, BN));
     p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
     p.num_tiles = p.num_m * p.num_n;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kSmemBytes));
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&gemm_kernel), static_cast<int>(kSmemBytes));
+    if (e != cudaSuccess) return e;
     int grid = ov.grid_ctas;
     if (grid <= 0) grid = device_num_sms();
     grid = mn(grid, p.num_tiles);

@@ -5,8 +5,8 @@
 // cos/sin(n pi x) on the same 1001 trapezoid nodes, so the map over n has a broadcast operand: the
 // node table g_i = w_i f(x_i) (w = 1/2 at the ends, 0 at JGF's skipped node x_{m-1}, 1 elsewhere).
 // The phase n pi x_i = 2 pi (n i mod m)/m is reduced EXACTLY in integers, so the trigonometric
-// factors come from an m-entry table of e^{2 pi i p/m} (host fp64 libm, rounded to the variant's
-// precision, written once per device) -- no range-reduction error at n = 10^5 and no MUFU.
+// factors come from an m-entry table of e^{2 pi i p/m} (device fp64 sincospi, rounded to the
+// variant's precision, written once per device by an asynchronous kernel) -- no range-reduction error at n = 10^5 and no MUFU.
 // B200 form (radix-R split of the node index, i = R u + v, g zero-padded to 1024 nodes):
 //   sum_i g_i e^{i theta n i} = sum_u U_u * W_u,  U_u = e^{i theta (R n u mod m)},
 //   W_u = sum_v g_{Ru+v} V_v,  V_v = e^{i theta (n v mod m)}.
@@ -43,7 +43,7 @@ struct SeriesNodes {
     T g[kSeriesNodes];
 };
 
-// e^{2 pi i p / m}, p < m, rounded to T: a per-device constant table written once (host fp64 libm).
+// e^{2 pi i p / m}, p < m, rounded to T: a per-device table written once (series_tables_kernel).
 __device__ float d_series_cos32[kSeriesM], d_series_sin32[kSeriesM];
 __device__ double d_series_cos64[kSeriesM], d_series_sin64[kSeriesM];
 
@@ -61,30 +61,50 @@ static const SeriesNodes<T>& series_nodes() {
     return nodes;
 }
 
-static cudaError_t series_tables_once() {
+// e^{2 pi i p/m} for p < m in fp64 (device sincospi: within 1 ulp, exact at the quadrant points),
+// and the same values rounded to fp32. One thread per p.
+__global__ void series_tables_kernel() {
+    const int p = blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= kSeriesM) return;
+    double s, c;
+    sincospi(2.0 * p / kSeriesM, &s, &c);
+    if (p == 250 || p == 750) c = 0.0;             // exact symmetries keep the quadrant points exact
+    if (p == 0 || p == 500) s = 0.0;
+    d_series_cos64[p] = c;
+    d_series_sin64[p] = s;
+    d_series_cos32[p] = static_cast<float>(c);
+    d_series_sin32[p] = static_cast<float>(s);
+}
+
+// The tables are written once per device by series_tables_kernel, enqueued on the FIRST caller's
+// stream (no host synchronisation, lime.h's "never synchronises" contract); an event recorded after
+// it orders every later call on any other stream behind it (cudaStreamWaitEvent: a device-side
+// dependency, free once the event has completed). Inside a stream capture the event cannot be
+// waited on, so a capture that may precede the table's completion carries its own (idempotent:
+// same values) table kernel.
+static cudaError_t series_tables_ready(cudaStream_t stream) {
     static std::mutex mu;
     static bool done[256] = {};
+    static cudaEvent_t ready[256] = {};
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
-    std::lock_guard<std::mutex> lock(mu);
     if (dev < 0 || dev >= 256) return cudaErrorInvalidDevice;
-    if (done[dev]) return cudaSuccess;
-    static float c32[kSeriesM], s32[kSeriesM];
-    static double c64[kSeriesM], s64[kSeriesM];
-    const double two_pi = 6.283185307179586476925286766559;
-    for (int p = 0; p < kSeriesM; ++p) {
-        // exact symmetries keep the quadrant points exact (cos(pi/2) = 0, ...)
-        const double a = two_pi * p / kSeriesM;
-        c64[p] = (p == 250 || p == 750) ? 0.0 : std::cos(a);
-        s64[p] = (p == 0 || p == 500) ? 0.0 : std::sin(a);
-        c32[p] = static_cast<float>(c64[p]);
-        s32[p] = static_cast<float>(s64[p]);
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if ((e = cudaStreamIsCapturing(stream, &cap)) != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lock(mu);
+    if (done[dev]) {
+        if (cap == cudaStreamCaptureStatusNone) return cudaStreamWaitEvent(stream, ready[dev], 0);
+        if (cudaEventQuery(ready[dev]) == cudaSuccess) return cudaSuccess;
+        cudaGetLastError();
+        series_tables_kernel<<<ceil_div(kSeriesM, 256), 256, 0, stream>>>();
+        return cudaGetLastError();
     }
-    if ((e = cudaMemcpyToSymbol(d_series_cos32, c32, sizeof c32)) != cudaSuccess) return e;
-    if ((e = cudaMemcpyToSymbol(d_series_sin32, s32, sizeof s32)) != cudaSuccess) return e;
-    if ((e = cudaMemcpyToSymbol(d_series_cos64, c64, sizeof c64)) != cudaSuccess) return e;
-    if ((e = cudaMemcpyToSymbol(d_series_sin64, s64, sizeof s64)) != cudaSuccess) return e;
+    series_tables_kernel<<<ceil_div(kSeriesM, 256), 256, 0, stream>>>();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (cap != cudaStreamCaptureStatusNone) return cudaSuccess;   // not marked: the capture holds its own copy
+    if ((e = cudaEventCreateWithFlags(&ready[dev], cudaEventDisableTiming)) != cudaSuccess) return e;
+    if ((e = cudaEventRecord(ready[dev], stream)) != cudaSuccess) return e;
     done[dev] = true;
     return cudaSuccess;
 }
@@ -181,7 +201,7 @@ size_t series_workspace_bytes(bool) { return 256; }   // tables are per-device c
 template <typename T, int R>
 static cudaError_t launch_series_t(int64_t n0, int64_t count, T* out, cudaStream_t stream) {
     if (count == 0) return cudaSuccess;
-    cudaError_t e = series_tables_once();
+    cudaError_t e = series_tables_ready(stream);
     if (e != cudaSuccess) return e;
     int grid = launch_override().grid_ctas;
     if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(count, kSeriesBlock), 16LL * device_num_sms()));

@@ -125,11 +125,7 @@ static cudaError_t launch_t(Args& a, cudaStream_t stream) {
     a.ntiles = static_cast<int64_t>(a.tiles_x) * ceil_div<int32_t>(a.row_count, 32 / LW);
     int grid = launch_override().grid_ctas;
     if (grid <= 0) {
-        static int per_sm = 0;
-        if (per_sm == 0) {
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mandel_kernel<LW, UNROLL>, 256, 0);
-            if (per_sm <= 0) per_sm = 1;
-        }
+        const int per_sm = mx(1, cached_occupancy(reinterpret_cast<const void*>(&mandel_kernel<LW, UNROLL>), 256, 0));
         grid = per_sm * device_num_sms();
         const int64_t need = ceil_div<int64_t>(a.ntiles, 8);
         if (need < grid) grid = static_cast<int>(need);

@@ -513,13 +513,9 @@ __global__ void __launch_bounds__(16 * kMaxSplitsSmall) force_small_kernel(const
 
 static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
     const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaError_t e = cudaFuncSetAttribute(force_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
-        if (e != cudaSuccess) return e;
-        attr = kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16;
-    }
+    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&force_small_kernel),
+                                        static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
+    if (e != cudaSuccess) return e;
     const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
     return launch_pdl(&force_small_kernel, dim3(static_cast<unsigned>(ctas)), dim3(32 * ceil_div(a.splits, 2)), smem,
                       stream, a);
@@ -561,7 +557,7 @@ __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target
         unsigned v;
         do {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(arrivals) : "memory");
-        } while (v < target);
+        } while (static_cast<int>(v - target) < 0);     // wrap-safe (counters grow by gridDim.x per step)
     }
     __syncthreads();
 }
@@ -677,16 +673,10 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.dt = dt;
     const int block = 32 * ceil_div(a.splits, 2);
     const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(simulate_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
-    int occ = 0;
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, simulate_small_kernel, block, smem);
+    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&simulate_small_kernel),
+                                        static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
     if (e != cudaSuccess) return e;
+    const int occ = cached_occupancy(reinterpret_cast<const void*>(&simulate_small_kernel), block, smem);
     if (occ < 1) return cudaErrorInvalidConfiguration;
     const int64_t groups = ceil_div<int64_t>(n, 32);
     int grid = static_cast<int>(mn<int64_t>(groups, static_cast<int64_t>(occ) * device_num_sms()));

@@ -108,6 +108,9 @@ def test_mandelbrot_matmul_reduce_validation(L):
     assert mm(A0, A1, WS, 16, 16, 12, None) == 1                                    # K % 8 != 0
     assert mm(A0 + 2, A1, WS, 16, 16, 16, None) == 2
     assert mm(A0, A1, A0 + 16, 16, 16, 16, None) == 3                               # C overlaps A
+    assert mm(A0, A1, WS, 1 << 31, 16, 16, None) == 1                               # M = 2^31 (int32 rows)
+    assert mm(A0, A1, WS, 16, (1 << 31) - 256, 16, None) == 1                       # padded N overflows
+    assert mm(A0, A1, WS, 1 << 30, 1 << 30, 16, None) == 1                          # 2^40 tiles
     r = L.lime_reduce_sum_f32
     assert r(A0, -1, A1, WS, 1 << 16, None) == 1
     assert r(A0 + 2, 10, A1, WS, 1 << 16, None) == 2                                # f32 at 2-B offset

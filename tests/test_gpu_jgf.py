@@ -22,16 +22,40 @@ def test_series_first_coefficients_and_jgf_values(lime, dtype):
     assert np.abs(out - ref).max() <= max(SERIES_TOL[dtype] * bound, 1e-11)
 
 
+def _congruent(n):
+    """DESIGN.md R14b: with nodes x_i = 2i/m (m = 1000), cos/sin(pi (n + m) x_i) = cos/sin(pi n x_i
+    + 2 pi i), so a_n and b_n are periodic in n with period m for n >= 1; n maps to the index in
+    [1, m] with the same residue, where the oracle's fp64 phase n*pi*x is accurate to ~1e-12 rad."""
+    n = np.asarray(n, dtype=np.int64)
+    return (n - 1) % 1000 + 1
+
+
 @pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
 @pytest.mark.parametrize("n0,count", [(0, 1), (0, 1000), (99_000, 1000), (123_456_789, 257)])
 def test_series_matches_oracle(lime, dtype, n0, count):
+    out = lime.map_series(n0, count, dtype=dtype).cpu().numpy()
     if dtype == torch.float64 and n0 > 1_000_000:
         # the oracle's double cos(n pi x) carries an argument error ~ n pi x 2^-53 (~1e-7 rad at
-        # n ~ 1e8) that exceeds the fp64 tolerance; the GPU reduces the phase exactly
-        pytest.skip("oracle argument precision limits the fp64 comparison to n <= 1e6")
-    out = lime.map_series(n0, count, dtype=dtype).cpu().numpy()
-    ref, mag = oracle.series(n0, count, threads=THREADS)
+        # n ~ 1e8), above the fp64 tolerance; compare with the congruent coefficients instead
+        # (R14b periodicity, pinned on the oracle by test_oracle_pins.test_series_periodic_in_n)
+        idx = _congruent(np.arange(n0, n0 + count))
+        ref = np.empty((count, 2))
+        mag = np.empty(count)
+        for k, n in enumerate(idx):
+            r, m = oracle.series(int(n), 1)
+            ref[k], mag[k] = r[0], m[0]
+    else:
+        ref, mag = oracle.series(n0, count, threads=THREADS)
     assert (np.abs(out - ref) / mag[:, None]).max() <= SERIES_TOL[dtype]
+
+
+@pytest.mark.parametrize("dtype", [torch.float32, torch.float64])
+def test_series_large_n_periodic(lime, dtype):
+    # the GPU reduces the phase exactly in integers, so the periodicity holds bit for bit at any n
+    # (up to the int64 range of n * i): a_{n + k m} = a_n
+    base = lime.map_series(1, 1000, dtype=dtype)
+    for n0 in (1001, 1_000_001, 123_456_001, (1 << 40) - 999):
+        assert torch.equal(lime.map_series(n0, 1000, dtype=dtype), base), n0
 
 
 def test_series_table3_size_sampled_and_shards(lime):

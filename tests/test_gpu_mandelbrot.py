@@ -37,14 +37,16 @@ def test_cyclic_shards(lime):
 
 
 def test_full_frame_config3(lime):
+    # SURVEY.md §8(c) C-mandelbrot pin 4: the whole 8192^2 frame of config 3, element by element,
+    # against the oracle (threaded over host cores by interleaved rows; every row is still the plain
+    # single-threaded C loop), plus the frame checksum and determinism.
     f = golden("mandelbrot_points.json")["frame"]
     W, H = f["width"], f["height"]
     gpu = lime.map_mandelbrot(W, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"]).cpu().numpy()
+    ref = oracle.mandelbrot(W, H, 0, 1, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"],
+                            threads=os.cpu_count() or 1)
+    bad = np.argwhere(gpu != ref)
+    assert bad.size == 0, (len(bad), bad[:8].tolist())
     assert int(gpu.sum(dtype=np.int64)) == f["checksum"]
-    assert np.array_equal(gpu[1:4096], gpu[8191:4096:-1])            # mirror symmetry
-    rows = np.random.default_rng(3).choice(H, 48, replace=False)
-    for r in rows:
-        ref = oracle.mandelbrot(W, H, int(r), 1, 1, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"])
-        assert np.array_equal(gpu[r], ref[0]), r
     again = lime.map_mandelbrot(W, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"]).cpu().numpy()
     assert np.array_equal(gpu, again)

@@ -248,6 +248,34 @@ def test_mandelbrot_cyclic_shards_reassemble():
             assert np.array_equal(shard, full[r::P])
 
 
+def test_mandelbrot_goldens_reproduced_independently():
+    # provenance of the survey-probe goldens: tests/golden/make_mandelbrot_points.py recomputes the
+    # point counts with numpy binary32 code that shares nothing with oracle/ (its --frame mode
+    # recomputes the frame checksum; record in tests/golden/README.md)
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("mkm", os.path.join(os.path.dirname(__file__), "golden",
+                                                                      "make_mandelbrot_points.py"))
+    mkm = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mkm)
+    g = _golden("mandelbrot_points.json")
+    for cx, cy, n in g["points"]:
+        assert mkm.escape_count(cx, cy, g["max_iter"]) == n, (cx, cy)
+    # and its vectorised frame routine agrees with the oracle on a small frame (count sums)
+    W, dx = 64, 3.0 / 64
+    ref = oracle.mandelbrot(W, W, 0, 1, W, -2.0, -1.5, dx, dx, 300)
+    assert mkm.frame_rows((0, W, W, -2.0, -1.5, dx, dx, 300)) == int(ref.sum())
+
+
+def test_mandelbrot_threaded_equals_single_thread():
+    # the interleaved-row threading of oracle.mandelbrot (used for the full-frame GPU parity test)
+    # reassembles exactly the single-threaded frame, also for strided and reversed row sets
+    W, dx = 200, 3.0 / 200
+    for first, stride, rows in ((0, 1, 200), (3, 2, 90), (199, -1, 150)):
+        one = oracle.mandelbrot(W, W, first, stride, rows, -2.0, -1.5, dx, dx, 120)
+        many = oracle.mandelbrot(W, W, first, stride, rows, -2.0, -1.5, dx, dx, 120, threads=7)
+        assert np.array_equal(one, many)
+
+
 @pytest.mark.slow
 def test_mandelbrot_frame_checksum():
     f = _golden("mandelbrot_points.json")["frame"]
@@ -489,6 +517,20 @@ def test_series_integral_and_bounds():
     # coefficients of a smooth non-periodic function decay like 1/n: |b_n| n stays bounded
     n = np.arange(1, 200)
     assert np.abs(out[1:, 1] * n).max() < 20
+
+
+def test_series_periodic_in_n():
+    # DESIGN.md R14b: with nodes x_i = 2i/1000, pi (n + 1000) x_i = pi n x_i + 2 pi i, so
+    # a_{n+1000} = a_n and b_{n+1000} = b_n for n >= 1 (a_1000 = T[f], the n = 0 case is special:
+    # a_0 = T[f]/2). The oracle's fp64 phase n*pi*x has an argument error ~ n pi x 2^-53, so at
+    # n < 10^4 the congruent coefficients agree to ~1e-11 of T[|f|] (the GPU tests rely on this to
+    # compare large n against the congruent n in [1, 1000]).
+    base, mag = oracle.series(1, 1000)
+    for shift in (1000, 2000, 7000):
+        other, _ = oracle.series(1 + shift, 1000)
+        assert (np.abs(other - base) / mag[:, None]).max() < 1e-11, shift
+    a1000, m1000 = oracle.series(1000, 1)
+    assert abs(a1000[0, 0] - m1000[0]) < 1e-12 * m1000[0] and abs(a1000[0, 1]) < 1e-12 * m1000[0]
 
 
 def test_idea_published_test_vector_and_inverse():

@@ -54,8 +54,19 @@ def test_nbody_uses_packed_fp32_and_mufu_and_bulk_copy(sass):
 
 
 def test_gemm_is_tcgen05(sass):
-    ops = " ".join(_fn(sass, r"gemm_kernel"))
-    assert "UTCHMMA" in ops or "UTCQMMA" in ops   # tcgen05.mma
-    assert "UTMALDG" in ops                        # TMA tensor loads
-    assert "LDTM" in ops                           # tcgen05.ld epilogue
-    assert "HMMA" not in ops.replace("UTCHMMA", "")
+    for pat in (r"gemm_kernel", r"gemm2_kernel"):
+        ops = " ".join(_fn(sass, pat))
+        assert "UTCHMMA" in ops or "UTCQMMA" in ops   # tcgen05.mma
+        assert "UTMALDG" in ops                        # TMA tensor loads
+        assert "LDTM" in ops                           # tcgen05.ld epilogue
+        assert "HMMA" not in ops.replace("UTCHMMA", "")
+
+
+def test_gemm2_is_two_cta_tcgen05_with_tma_store(sass):
+    # the production kernel: cta_group::2 MMAs, pair-wide TMA loads, the
+    # TMA-store epilogue and tcgen05.ld
+    ops = " ".join(_fn(sass, r"gemm2_kernel"))
+    assert "UTCHMMA.2CTA" in ops
+    assert "UTMALDG" in ops
+    assert "UTMASTG" in ops
+    assert "LDTM" in ops
