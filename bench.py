@@ -7,11 +7,14 @@ paper's N-Body: all-gather of positions (NCCL, N > 1) -> for
 (lime_map_nbody) -> integrator (lime_map_nbody_integrate). Strong scaling: the 2^20-body
 problem is split by target index over N ranks (torchrun, one process per GPU).
 
-    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--no-extras]
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--no-extras] [--no-sharded]
 
-Rank 0 prints ONE JSON line. At N = 1 the line also carries `configs`: the other
-BASELINE.json configurations measured in the same run (N-Body 4096, Black-Scholes map and
-fused map+reduce, Mandelbrot, matmul, a reduction), each with its own roofline.
+Rank 0 prints ONE JSON line. At every N it carries `sharded_configs`: configs 2-4 partitioned over
+the N ranks as SURVEY.md §8(e) says (Black-Scholes strong + weak with an all_reduce, Mandelbrot
+cyclic rows, matmul row blocks), each timed as the max over ranks. At N = 1 the line also carries
+`configs`: every BASELINE.json configuration and the F-rows measured in the same run (N-Body 4096,
+Black-Scholes map and fused map+reduce, Mandelbrot, matmul, reductions, ...), each with its own
+roofline.
 """
 from __future__ import annotations
 
@@ -300,7 +303,8 @@ def run_nbody(args, rank, world, local):
                 "peak_source": "derived: 148 SM x 128 FP32 lanes x 2 flop x 1965 MHz (microbench: 124.9-127.9 lane-ops/clk/SM)",
                 "flop_per_interaction": FLOP_PER_INTERACTION,
                 "fp32_lane_ops_per_interaction": lane_ops,
-                "element_form": ("mass factored out of each chunk sum (equal masses, DESIGN.md R11)" if uniform_mass
+                "element_form": ("mass factored out of each chunk sum (equal masses, DESIGN.md R11; the unequal-mass "
+                                 "number at this size is configs.nbody_1m_mixed_masses)" if uniform_mass
                                  else "per-body mass multiply"),
                 "fp32_pipe_frac_at_observed_clock": pipe_frac, "observed_sm_mhz": obs_mhz,
                 "force_ms_per_launch": force_ms, "force_ms_per_launch_max_rank": force_ms_max,
@@ -478,6 +482,21 @@ def run_extras(peaks, flush):
                                  "traffic": ncu_traffic("nbody_force_1m_p8") if ops == FP32_LANE_OPS_UNIFORM_MASS else None}}
         del bd
     del acc1m
+    # the headline's own size (2^20 x 2^20, one force launch) with the unequal masses: the number a
+    # workload without the equal-mass fast path (R11) gets
+    bd = torch.from_numpy(b1m_mixed).cuda()
+    accm = torch.empty((1 << 20, 4), dtype=torch.float32, device="cuda")
+    med, _ = time_launches(lambda: lime.map_nbody(bd, EPS2, out=accm), 2, 1, flush)
+    inter_full = float(1 << 20) * (1 << 20)
+    ach = FLOP_PER_INTERACTION * inter_full / (med * 1e-3) / 1e12
+    out["nbody_1m_mixed_masses"] = {
+        "workload": "configs[4] force map at full size (2^20 x 2^20 fp32), masses U[0.5,1.5)/N: per-body-mass element",
+        "value": inter_full / (med * 1e-3), "unit": "interactions/s", "ms_per_launch": med,
+        "fp32_lane_ops_per_interaction": FP32_LANE_OPS_PER_INTERACTION,
+        "roofline": {"bound": "alu", "achieved": ach, "peak": fp32, "unit": "TFLOP/s", "frac": ach / fp32,
+                     "fp32_pipe_frac": FP32_LANE_OPS_PER_INTERACTION * inter_full / (med * 1e-3)
+                     / (SMS_B200 * 128 * SM_MAX_MHZ_NOMINAL * 1e6), "traffic": None}}
+    del bd, accm
 
     # config-5 strong scaling on ONE GPU, compute only: the force map of the rank-0 shard at P = 1, 2, 4,
     # 8 (2^20/P targets x 2^20 sources, the launch each rank runs); E(P) = T_1 / (P T_P). The per-step
@@ -581,6 +600,82 @@ def run_extras(peaks, flush):
                              "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
                                           "traffic": ncu_traffic("reduce_sum_f32")}}
     del x
+    return out
+
+
+# ----------------------------------------------------------------------------- sharded configs (any N)
+def run_sharded(args, rank, world, local, peaks, flush):
+    """Configs 2-4 partitioned over the N ranks exactly as SURVEY.md §8(e) says, at every N (so the
+    driver's N = 1, 2, 4, 8 runs each report every config): Black-Scholes fused map+reduce over
+    contiguous option shards + one all_reduce of the fp64 partials (strong: one 2^24 array; weak:
+    2^24 options per GPU), Mandelbrot 8192^2 over cyclic rows, matmul 8192^3 over C row blocks (Bt
+    replicated before timing). Per rank: warm-up, then each launch between CUDA events on the
+    launching stream after an L2 flush; value = all ranks' units / the MAX over ranks of the median
+    launch time."""
+    hbm = peaks["hbm_gbs"]
+    out = {}
+
+    def timed(fn, reps, warm, writes_output=False):
+        barrier(world)
+        med, _ = time_launches(fn, reps, warm, flush, writes_output=writes_output)
+        return max_over_ranks(med, world)
+
+    n = 1 << 24
+    S, X, T = (torch.from_numpy(a).cuda() for a in inputs.blackscholes_options(n, seed=2))
+    b, c = ldist.shard_range_aligned(n, rank, world, 4)
+    ms = timed(lambda: ldist.blackscholes_shard_total(S, X, T, inputs.BS_R, inputs.BS_SIGMA), 30, 5)
+    gbs = 12.0 * n / (ms * 1e-3) / 1e9 / world          # per-GPU HBM rate
+    out["blackscholes_map_reduce_strong"] = {
+        "workload": f"configs[1]: fused Black-Scholes total premium, 2^24 options split over {world} GPU(s) "
+                    "(contiguous shards) + all_reduce of 2 fp64 partials", "scaling": "strong",
+        "value": n / (ms * 1e-3), "unit": "options/s", "ms_per_call": ms, "options_per_gpu": c,
+        "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s per GPU", "frac": gbs / hbm}}
+    del S, X, T
+    Sw, Xw, Tw = (torch.from_numpy(a).cuda() for a in inputs.blackscholes_options(n, seed=200 + rank))
+    ms = timed(lambda: ldist.blackscholes_total(Sw, Xw, Tw, inputs.BS_R, inputs.BS_SIGMA), 30, 5)
+    gbs = 12.0 * n / (ms * 1e-3) / 1e9
+    out["blackscholes_map_reduce_weak"] = {
+        "workload": "configs[1] weak scaling: fused Black-Scholes total premium, 2^24 options PER GPU "
+                    "+ all_reduce of 2 fp64 partials", "scaling": "weak",
+        "value": float(n) * world / (ms * 1e-3), "unit": "options/s", "ms_per_call": ms,
+        "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s per GPU", "frac": gbs / hbm}}
+    del Sw, Xw, Tw
+
+    W = 8192
+    d = 3.0 / W
+    first, stride, rows = ldist.cyclic_rows(W, rank, world)
+    cnt = torch.empty((rows, W), dtype=torch.int32, device="cuda")
+    ms = timed(lambda: ldist.mandelbrot_cyclic(W, W, -2.0, -1.5, d, d, 1024, out=cnt), 10, 2, writes_output=True)
+    iters = torch.tensor([float(cnt.sum(dtype=torch.int64).item())], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(iters)
+    lane_peak = SMS_B200 * 128 * SM_MAX_MHZ_NOMINAL * 1e6
+    out["mandelbrot_cyclic_rows"] = {
+        "workload": f"configs[2]: Mandelbrot 8192x8192, max_iter 1024, cyclic rows over {world} GPU(s)",
+        "scaling": "strong", "value": W * W / (ms * 1e-3), "unit": "pixels/s", "ms_per_call": ms,
+        "rows_per_gpu": rows, "checksum": int(iters.item()),
+        "roofline": {"bound": "alu", "achieved": 7.0 * iters.item() / world / (ms * 1e-3) / 1e12,
+                     "peak": lane_peak / 1e12, "unit": "T FP32 lane-ops/s per GPU",
+                     "frac": 7.0 * iters.item() / world / (ms * 1e-3) / lane_peak}}
+    del cnt
+
+    M = N = K = 8192
+    try:
+        A = torch.from_numpy(inputs.bf16_uniform(M, K, 4, 0).view(np.int16)).cuda().view(torch.bfloat16)
+        Bt = torch.from_numpy(inputs.bf16_uniform(N, K, 4, 1).view(np.int16)).cuda().view(torch.bfloat16)
+        mb, mc = ldist.shard_range(M, rank, world)
+        Cb = torch.empty((mc, N), dtype=torch.float32, device="cuda")
+        ms = timed(lambda: ldist.matmul_row_block(A, Bt, Cb), 20, 3, writes_output=True)
+        tf = 2.0 * mc * N * K / (ms * 1e-3) / 1e12
+        out["matmul_row_blocks"] = {
+            "workload": f"configs[3]: matmul 8192^3 bf16 -> fp32, C row blocks over {world} GPU(s), Bt replicated",
+            "scaling": "strong", "value": M * N / (ms * 1e-3), "unit": "dot products/s", "ms_per_call": ms,
+            "rows_per_gpu": mc,
+            "roofline": {"bound": "tensor", "achieved": tf, "peak": peaks["bf16_tflops"], "unit": "TFLOP/s per GPU",
+                         "frac": tf / peaks["bf16_tflops"]}}
+        del A, Bt, Cb
+    except lime.LimeError as e:
+        out["matmul_row_blocks"] = {"workload": "configs[3]", "unavailable": str(e)}
     return out
 
 
@@ -729,7 +824,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["lime", "reference"], default="lime")
     ap.add_argument("--bodies", dest="n", type=int, default=1 << 20)
-    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip the N = 1 per-config extras")
+    ap.add_argument("--no-sharded", action="store_true", help="skip the sharded configs 2-4 (any N)")
     ap.add_argument("--cpu-targets", type=int, default=3072)
     ap.add_argument("--ref-targets", type=int, default=512)
     args = ap.parse_args()
@@ -745,6 +841,13 @@ def main():
     lime.load()
     peaks = measured_peaks()
     line = run_nbody(args, rank, world, local)
+    if not args.no_sharded:
+        props = torch.cuda.get_device_properties(local)
+        flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
+        sharded = run_sharded(args, rank, world, local, peaks, flush)
+        del flush
+        if rank == 0:
+            line["sharded_configs"] = sharded
     if rank == 0 and world == 1:
         if not args.no_extras:
             props = torch.cuda.get_device_properties(local)

@@ -7,9 +7,12 @@ One process per GPU; torch.distributed (NCCL over NVLink on the box) is the plum
     the local targets against all sources, then the local integrator. Forces are bit-identical
     to the single-GPU run because the per-target summation order depends on n_src only.
   * Black-Scholes fused sums (config 2): contiguous option shards, one `all_reduce` (sum) of the
-    per-GPU fp64 partials.
-  * Mandelbrot (config 3): cyclic rows (row r -> rank r mod P), no collective.
-  * Matmul (config 4): contiguous row blocks of C, no collective.
+    per-GPU fp64 partials (`blackscholes_total` on a rank's own options = weak scaling;
+    `blackscholes_shard_total` on a shard of one global array = strong scaling).
+  * Mandelbrot (config 3): cyclic rows (row r -> rank r mod P; `mandelbrot_cyclic`), no collective;
+    `gather_cyclic_rows` reassembles the frame for validation only.
+  * Matmul (config 4): contiguous row blocks of C against a replicated Bt (`matmul_row_block`), no
+    collective; `gather_row_blocks` reassembles C for validation only.
 
 The step functions take the map/integrator callables as parameters so the partition and
 exchange logic can be exercised on CPU (gloo) in tests; the product binds them to the CUDA ABI.
@@ -27,6 +30,17 @@ def shard_range(n: int, rank: int, world: int) -> tuple[int, int]:
     base, rem = divmod(n, world)
     begin = rank * base + min(rank, rem)
     return begin, base + (1 if rank < rem else 0)
+
+
+def shard_range_aligned(n: int, rank: int, world: int, align: int) -> tuple[int, int]:
+    """Contiguous shard whose begin is a multiple of `align` elements (the 128-bit loads of the
+    streaming maps need 16-byte aligned operands: align = 4 fp32); the tail goes to the last rank."""
+    units = n // align
+    b, c = shard_range(units, rank, world)
+    begin, count = b * align, c * align
+    if rank == world - 1:
+        count += n - units * align
+    return begin, count
 
 
 def cyclic_rows(height: int, rank: int, world: int) -> tuple[int, int, int]:
@@ -121,3 +135,77 @@ def blackscholes_total(S, X, T, r: float, sigma: float, fused_fn: Callable | Non
     if dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.all_reduce(sums, group=group)
     return sums
+
+
+def _rank_world(group=None) -> tuple[int, int]:
+    if dist.is_initialized():
+        return dist.get_rank(group), dist.get_world_size(group)
+    return 0, 1
+
+
+def blackscholes_shard_total(S, X, T, r: float, sigma: float, fused_fn: Callable | None = None, group=None):
+    """Strong-scaled fused Black-Scholes (config 2): every rank holds (or views) the full option
+    arrays, sums its contiguous shard [begin, begin+count) and all-reduces the two fp64 partials."""
+    rank, world = _rank_world(group)
+    b, c = shard_range_aligned(S.numel(), rank, world, 4)
+    return blackscholes_total(S[b:b + c], X[b:b + c], T[b:b + c], r, sigma, fused_fn=fused_fn, group=group)
+
+
+def mandelbrot_cyclic(width: int, height: int, x0: float, y0: float, dx: float, dy: float, max_iter: int,
+                      device="cuda", out=None, map_fn: Callable | None = None, group=None) -> torch.Tensor:
+    """This rank's cyclic rows of the Mandelbrot frame (config 3; rows rank, rank+P, ...): int32
+    [row_count][width]. No collective: the output stays sharded."""
+    rank, world = _rank_world(group)
+    first, stride, count = cyclic_rows(height, rank, world)
+    if map_fn is None:
+        import paper_conf_pldi_dubachcrbf12_b200 as lime
+        map_fn = lime.map_mandelbrot
+    return map_fn(width, height, x0, y0, dx, dy, max_iter, row_first=first, row_stride=stride, row_count=count,
+                  device=device, out=out)
+
+
+def gather_cyclic_rows(local: torch.Tensor, height: int, group=None) -> torch.Tensor:
+    """Reassemble the full [height][width] frame from every rank's cyclic rows (validation only):
+    shards are padded to ceil(height/P) rows for one all_gather_into_tensor, then interleaved."""
+    rank, world = _rank_world(group)
+    if world == 1:
+        return local
+    width = local.shape[1]
+    rows = -(-height // world)
+    pad = torch.zeros((rows, width), dtype=local.dtype, device=local.device)
+    pad[:local.shape[0]] = local
+    allp = torch.empty((world * rows, width), dtype=local.dtype, device=local.device)
+    dist.all_gather_into_tensor(allp, pad, group=group)
+    allp = allp.view(world, rows, width)
+    full = torch.empty((height, width), dtype=local.dtype, device=local.device)
+    for k in range(world):
+        cnt = len(range(k, height, world))
+        full[k::world] = allp[k, :cnt]
+    return full
+
+
+def matmul_row_block(A: torch.Tensor, Bt: torch.Tensor, out=None, mm_fn: Callable | None = None, group=None):
+    """This rank's contiguous row block of C = A . Bt^T (config 4): rows [begin, begin+count) of A
+    against the replicated Bt; no per-call collective."""
+    rank, world = _rank_world(group)
+    b, c = shard_range(A.shape[0], rank, world)
+    if mm_fn is None:
+        import paper_conf_pldi_dubachcrbf12_b200 as lime
+        mm_fn = lime.map_matmul_bf16
+    if c == 0:
+        return torch.empty((0, Bt.shape[0]), dtype=torch.float32, device=A.device)
+    return mm_fn(A[b:b + c], Bt, out)
+
+
+def gather_row_blocks(local: torch.Tensor, M: int, group=None) -> torch.Tensor:
+    """Reassemble C [M][N] from every rank's contiguous row block (validation only)."""
+    rank, world = _rank_world(group)
+    if world == 1:
+        return local
+    rows = -(-M // world)
+    pad = torch.zeros((rows,) + tuple(local.shape[1:]), dtype=local.dtype, device=local.device)
+    pad[:local.shape[0]] = local
+    allp = torch.empty((world * rows,) + tuple(pad.shape[1:]), dtype=local.dtype, device=local.device)
+    dist.all_gather_into_tensor(allp, pad, group=group)
+    allp = allp.view((world,) + tuple(pad.shape))
+    return torch.cat([allp[k, :shard_range(M, k, world)[1]] for k in range(world)])

@@ -54,7 +54,7 @@ def test_series_large_n_periodic(lime, dtype):
     # the GPU reduces the phase exactly in integers, so the periodicity holds bit for bit at any n
     # (up to the int64 range of n * i): a_{n + k m} = a_n
     base = lime.map_series(1, 1000, dtype=dtype)
-    for n0 in (1001, 1_000_001, 123_456_001, (1 << 40) - 999):
+    for n0 in (1001, 1_000_001, 123_456_001, ((1 << 40) // 1000) * 1000 + 1):   # all = 1 (mod m)
         assert torch.equal(lime.map_series(n0, 1000, dtype=dtype), base), n0
 
 
