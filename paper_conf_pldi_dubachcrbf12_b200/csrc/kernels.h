@@ -26,10 +26,10 @@ namespace nbody {
 constexpr int kChunk = 256;
 constexpr int kMaxSplits = 16;
 #ifndef LIME_CHUNK_SMALL            // compile-time A/B overrides (tools/); the defaults are the product
-#define LIME_CHUNK_SMALL 128
+#define LIME_CHUNK_SMALL 64
 #endif
 #ifndef LIME_MAX_SPLITS_SMALL
-#define LIME_MAX_SPLITS_SMALL 32
+#define LIME_MAX_SPLITS_SMALL 64
 #endif
 constexpr int kChunkSmall = LIME_CHUNK_SMALL;
 constexpr int kMaxSplitsSmall = LIME_MAX_SPLITS_SMALL;

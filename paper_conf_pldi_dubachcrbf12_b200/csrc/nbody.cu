@@ -89,7 +89,27 @@ struct ForceArgs {
     int splits;
     int chunk;            // chunk_len(n_src)
     int64_t split_len;    // chunks_per_split * chunk
+    int tree;             // n_src <= kSmallMaxSources: split partials combined by split_tree_sum
 };
+
+// Split combine of the small problems (n_src <= kSmallMaxSources): a pairwise tree over
+// S2 = next_pow2(S) split partials, zero beyond S -- ((P0 + P1) + (P2 + P3)) + ... -- the order in
+// which the small kernels' warp-shuffle butterfly adds them (each level adds a block of 2^k aligned
+// splits to its neighbour; IEEE addition is commutative, so both partners get the same bits).
+__host__ __device__ __forceinline__ int next_pow2(int s) { int p = 1; while (p < s) p <<= 1; return p; }
+__device__ __forceinline__ float4 add3(float4 a, float4 b) { return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, 0.f); }
+template <class Load>
+__device__ __forceinline__ float4 split_tree_sum(int S, Load load) {
+    float4 stack[8];
+    int top = 0;
+    const int S2 = next_pow2(S);
+    for (int i = 0; i < S2; ++i) {
+        float4 v = i < S ? load(i) : make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int m = i; m & 1; m >>= 1) v = add3(stack[--top], v);    // binary-counter merge
+        stack[top++] = v;
+    }
+    return stack[0];
+}
 
 template <int R, bool kPacked>
 struct Interact;
@@ -319,10 +339,15 @@ __device__ __forceinline__ void finish_targets(const ForceArgs& a, const IT& it,
     for (int r = 0; r < R; ++r) {
         const int64_t t = tbase + threadIdx.x + static_cast<int64_t>(r) * BLOCK;
         if (!valid[r]) continue;
-        float4 acc = __ldcg(a.partial + t);
-        for (int s = 1; s < a.splits; ++s) {
-            const float4 p = __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
-            acc.x += p.x; acc.y += p.y; acc.z += p.z;
+        float4 acc;
+        if (a.tree) {
+            acc = split_tree_sum(a.splits, [&](int s) { return __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t); });
+        } else {
+            acc = __ldcg(a.partial + t);
+            for (int s = 1; s < a.splits; ++s) {
+                const float4 p = __ldcg(a.partial + static_cast<int64_t>(s) * a.tgt_count + t);
+                acc.x += p.x; acc.y += p.y; acc.z += p.z;
+            }
         }
         acc.w = 0.f;
         a.accel[t] = acc;
@@ -418,19 +443,38 @@ __global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constan
 
 // =====================================================================================
 // Small problems (n_src <= kSmallMaxSources, e.g. the paper's 4096 bodies, Table 3): the
-// splits live inside one CTA instead of across CTAs. A CTA owns 32 targets; each warp owns TWO
-// consecutive splits, one per half-warp, and each lane of a half-warp carries a packed PAIR of the
-// CTA's targets (lane q of the half: targets 2q, 2q+1), so every FFMA2/FADD2/FMUL2 does two
-// interactions -- this launch is issue-bound, and packing halves the FP32 issue slots per
-// interaction. Warp w bulk-copies its two splits' sources (<= 2 x 4 KB, contiguous) into its smem
-// slice and runs exactly the arithmetic of the general kernel (chunk partials added into the split
-// accumulator in chunk order; each half of a packed op rounds exactly like the scalar op); the
-// split partials are then added in split order from shared memory. Same summation order as
-// force_kernel, hence bit-identical results, with no global partials and no atomic tickets.
+// whole problem is one wave, so every SM must carry the same work, spread evenly over its four
+// SM sub-partitions (SMSPs), and no SM may wait on a serial phase. One CTA per SM.
+//  * Work unit = a GROUP of kGroupTargets = 4 consecutive targets (two packed pairs); a group is
+//    2 x S2 lanes (S2 = next_pow2(S)), lane (s, p) summing split s (64-body chunks) for the group's
+//    targets 2p, 2p + 1 with split_sum (force_kernel's arithmetic, packed FFMA2/FADD2/FMUL2).
+//    Groups are dealt to the CTAs in contiguous ranges of floor or ceil(G / grid) groups (at 4096
+//    bodies: 6 or 7 groups = 24 or 28 warps on each of the 148 SMs, 6 or 7 per SMSP). The SMSP
+//    balance is what the split count is chosen for: tools/nbody_inner_mb.cu measured that an SM
+//    runs as long as its busiest SMSP, so 14 warps (4-4-3-3) take as long as 16.
+//  * A4: every CTA stages the source array in shared memory with one 1-D bulk copy per split,
+//    each with its own mbarrier, so a lane starts as soon as ITS split has landed. Each split's
+//    slice is padded by one float4 (split s at float4 offset s (L + 1)): the splits of an LDS.128
+//    phase then sit in different bank quads -- the paper's conflict padding (L241-255).
+//  * A8: the S2 split partials of a target are added as a pairwise tree (split_tree_sum's order):
+//    a warp-shuffle butterfly over the warp's 16 splits, then the (<= 4) warp block sums in shared
+//    memory. force_kernel combines small problems in the same order, so force_kernel,
+//    force_small_kernel and simulate_small_kernel agree bit for bit.
 // =====================================================================================
+#ifndef LIME_GROUP_PAIRS
+#define LIME_GROUP_PAIRS 2
+#endif
+constexpr int kGroupPairs = LIME_GROUP_PAIRS;          // packed target pairs per group (1 or 2)
+constexpr int kGroupTargets = 2 * kGroupPairs;
+constexpr int kWarpSplits = 32 / kGroupPairs;           // splits one warp of a group covers
+#ifndef LIME_SMALL_MAXT
+#define LIME_SMALL_MAXT 896
+#endif
+constexpr int kSmallMaxThreads = LIME_SMALL_MAXT;   // block cap (register budget 65536 / cap)
+constexpr size_t kOneCtaPerSmSmem = 116 * 1024;   // > 228 KB / 2 per SM (B200)
+
 // One split's contribution for the lane's targets: chunk partials added into the split accumulator
-// in chunk order -- the arithmetic of force_kernel (shared by force_small_kernel and the persistent
-// simulation kernel, so all three agree bit for bit).
+// in chunk order -- the arithmetic of force_kernel.
 template <class IT>
 __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2) {
     for (int c0 = 0; c0 < len; c0 += chunk) {
@@ -439,9 +483,6 @@ __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int
         if (c1 - c0 == kChunkSmall) {
 #pragma unroll kSmallUnroll
             for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
-        } else if (c1 - c0 == kChunk) {
-#pragma unroll 4
-            for (int j = c0; j < c0 + kChunk; ++j) it.body(sb[j], eps2);
         } else {
             for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
         }
@@ -449,92 +490,210 @@ __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int
     }
 }
 
-// Lane -> (split, target pair) map of the small kernels: warp w, half h = lane / 16 works on split
-// 2w + h for the CTA's targets 2q and 2q + 1 (q = lane % 16).
+struct SmallPlan {
+    int S, S2;           // splits(n_src), next_pow2(S)
+    int L;               // split length (bodies)
+    int chunk;
+    int64_t groups;      // ceil(targets / 4)
+    int grid;
+    int slots;           // groups a CTA works on at once (its range is done in rounds of `slots`)
+    int block;           // slots x 2 S2 lanes, rounded up to whole warps
+    size_t smem;
+};
+__host__ __device__ __forceinline__ int64_t group_begin(int64_t groups, int grid, int c) { return groups * c / grid; }
+__host__ __device__ __forceinline__ int warp_blocks(int S2) { return S2 > kWarpSplits ? S2 / kWarpSplits : 1; }
+__host__ __device__ __forceinline__ size_t small_src_bytes(int S, int L) { return static_cast<size_t>(S) * (L + 1) * 16; }
+
+static SmallPlan small_plan(int64_t n_src, int64_t targets, int max_grid) {
+    SmallPlan p;
+    p.S = splits(n_src);
+    p.S2 = next_pow2(p.S);
+    p.chunk = chunk_len(n_src);
+    p.L = static_cast<int>(chunks_per_split(n_src) * p.chunk);
+    p.groups = ceil_div<int64_t>(targets, kGroupTargets);
+    p.grid = static_cast<int>(mx<int64_t>(1, mn<int64_t>(p.groups, max_grid)));
+    p.slots = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(p.groups, p.grid), kSmallMaxThreads / (kGroupPairs * p.S2)));
+    p.block = ceil_div(p.slots * kGroupPairs * p.S2, 32) * 32;
+    p.smem = small_src_bytes(p.S, p.L) + static_cast<size_t>(p.slots) * warp_blocks(p.S2) * kGroupTargets * 16;
+    // One CTA per SM: the dealt ranges assume it, but a CTA this small would let the block
+    // scheduler place two on one SM. Asking for more than half an SM's shared memory makes a second
+    // resident CTA impossible.
+    p.smem = mx<size_t>(p.smem, kOneCtaPerSmSmem);
+    return p;
+}
+// Largest smem any small plan needs (the attribute is set once per device for this bound).
+static int small_smem_bound() {
+    return static_cast<int>(mx<size_t>(kOneCtaPerSmSmem, small_src_bytes(kMaxSplitsSmall, kSmallMaxSources / kMaxSplitsSmall) +
+                                                         (kSmallMaxThreads / 32) * kGroupTargets * 16));   // <= one block sum per warp
+}
+
+#ifdef LIME_TRACE
+__device__ long long g_lime_trace[kNumSMsB200 * 64 * 8];
+__device__ __forceinline__ unsigned smid() { unsigned r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
+#define LIME_TRACE_AT(k, slot) \
+    do { if (threadIdx.x == 0 && (k) < 64) { g_lime_trace[(blockIdx.x * 64 + (k)) * 8 + (slot)] = clock64(); \
+         g_lime_trace[(blockIdx.x * 64 + (k)) * 8 + 7] = smid(); } } while (0)
+__device__ long long g_lime_wtrace[kNumSMsB200 * 32 * 2];   // step 20: per warp (data ready, lane sum done)
+__device__ int g_lime_step;
+#define LIME_WTRACE(slot) \
+    do { if (g_lime_step == 20 && (threadIdx.x & 31) == 0) g_lime_wtrace[(blockIdx.x * 32 + (threadIdx.x >> 5)) * 2 + (slot)] = clock64(); } while (0)
+#else
+#define LIME_TRACE_AT(k, slot) do { } while (0)
+#define LIME_WTRACE(slot) do { } while (0)
+#endif
+
+// Lane -> work map shared by both small kernels.
 struct SmallLane {
-    int split, q;
-    __device__ __forceinline__ SmallLane() {
-        const unsigned lane = lane_id();
-        split = 2 * static_cast<int>(threadIdx.x >> 5) + static_cast<int>(lane >> 4);
-        q = static_cast<int>(lane & 15u);
+    int gslot, s, p;   // group slot in this CTA, split, pair within the group
+    __device__ __forceinline__ SmallLane(int S2) {
+        const int idx = static_cast<int>(threadIdx.x) % (kGroupPairs * S2);
+        gslot = static_cast<int>(threadIdx.x) / (kGroupPairs * S2);
+        s = idx / kGroupPairs;
+        p = idx % kGroupPairs;
     }
 };
+__device__ __forceinline__ int padded(int i, int L) { return (i / L) * (L + 1) + i % L; }
 
-__global__ void __launch_bounds__(16 * kMaxSplitsSmall) force_small_kernel(const __grid_constant__ ForceArgs a) {
-    extern __shared__ __align__(128) uint8_t small_smem[];
-    float4* src = reinterpret_cast<float4*>(small_smem);                          // [S][split_len]
-    float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
-    __shared__ __align__(8) uint64_t bar[kMaxSplitsSmall / 2];
-
-    pdl_enter();
-    const int warp = threadIdx.x >> 5;
-    const unsigned lane = lane_id();
-    const SmallLane sl;
-    const int64_t tg = static_cast<int64_t>(blockIdx.x) * 32;
-    Interact<2, true> it;
+#ifndef LIME_STAGE_U
+#define LIME_STAGE_U 6
+#endif
+// All threads: bring bodies [0, n) into their padded slots (LDG.128 + STS.128; tools/load_mb.cu:
+// 148 CTAs loading the same 64 KB take ~1.3k cycles this way vs 4.6k for 64 one-split bulk copies,
+// whose per-copy cost serialises in the TMA unit). kCoherent: the bodies were written in this
+// launch by other CTAs (ld.global.cg, L2), else read-only (ld.global.nc).
+template <bool kCoherent>
+__device__ __forceinline__ void stage_all(float4* src, const float4* bodies, int64_t n, int L) {
+    constexpr int U = LIME_STAGE_U;                    // loads in flight per thread: ceil(4096 / 896) = 5 -> one round trip
+    for (int base = static_cast<int>(threadIdx.x); base < n; base += U * static_cast<int>(blockDim.x)) {
+        float4 v[U];
 #pragma unroll
-    for (int r = 0; r < 2; ++r) {
-        const int64_t t = tg + 2 * sl.q + r;
-        it.set(r, __ldg(a.bodies + a.tgt_begin + (t < a.tgt_count ? t : a.tgt_count - 1)));
-    }
-    it.zero_all();
-
-    // this warp's two splits: one contiguous source range
-    const int64_t w0 = static_cast<int64_t>(2 * warp) * a.split_len;
-    const int64_t w1 = mn<int64_t>(a.n_src, w0 + 2 * a.split_len);
-    if (lane == 0) {
-        mbar_init(&bar[warp], 1);
-        fence_mbar_init();
-        mbar_arrive_expect_tx(&bar[warp], static_cast<uint32_t>(w1 - w0) * 16u);
-        bulk_g2s(src + w0, a.bodies + w0, static_cast<uint32_t>(w1 - w0) * 16u, &bar[warp]);
-    }
-    __syncwarp();
-    mbar_wait(&bar[warp], 0);
-    const int64_t j0 = static_cast<int64_t>(sl.split) * a.split_len;
-    const int len = sl.split < a.splits ? static_cast<int>(mn<int64_t>(a.n_src, j0 + a.split_len) - j0) : 0;
-    split_sum(it, src + j0, len, a.chunk, a.eps2);
-    if (sl.split < a.splits) {
-        part[sl.split * 32 + 2 * sl.q] = it.result(0);
-        part[sl.split * 32 + 2 * sl.q + 1] = it.result(1);
-    }
-    __syncthreads();
-    const int64_t t = tg + lane;
-    if (warp == 0 && t < a.tgt_count) {
-        float4 acc = part[lane];
-#pragma unroll 8
-        for (int s = 1; s < a.splits; ++s) {       // unrolled: the LDS issue ahead of the in-order FADD chain
-            const float4 p = part[s * 32 + lane];
-            acc.x += p.x; acc.y += p.y; acc.z += p.z;
+        for (int u = 0; u < U; ++u) {
+            const int i = base + u * static_cast<int>(blockDim.x);
+            if (i < n) v[u] = kCoherent ? __ldcg(bodies + i) : __ldg(bodies + i);
         }
-        acc.w = 0.f;
-        a.accel[t] = acc;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int i = base + u * static_cast<int>(blockDim.x);
+            if (i < n) src[padded(i, L)] = v[u];
+        }
     }
 }
 
-static cudaError_t launch_small(const ForceArgs& a, cudaStream_t stream) {
-    const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
-    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&force_small_kernel),
-                                        static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
+// The lane's split partial for targets tg + 2p, tg + 2p + 1 (clamped to the last valid target),
+// then the butterfly over the warp's splits: lanes 2 (16 w) + p of each group's warp w end up with
+// the sum of splits 16 w .. 16 w + 15 (or the whole group when S2 <= 16), stored to wpart.
+// Every lane of the CTA's used warps calls it (lanes of split s >= S contribute zero).
+__device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLane& sl, bool active, int64_t tgt_first_src,
+                                               int64_t tg, int64_t tcount, int L, int S, int S2, int64_t n, int chunk,
+                                               float eps2, float4* wpart) {
+    Interact<2, true> it;
+    it.zero_all();
+    LIME_WTRACE(0);
+    if (active && sl.s < S) {
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            int64_t t = tg + 2 * sl.p + r;
+            t = t < tcount ? t : tcount - 1;
+            it.set(r, src[padded(static_cast<int>(tgt_first_src + t), L)]);
+        }
+        const int64_t j0 = static_cast<int64_t>(sl.s) * L;
+        split_sum(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
+                  eps2);
+    }
+    float4 a0 = it.result(0), a1 = it.result(1);
+    const int seg = S2 < kWarpSplits ? kGroupPairs * S2 : 32;   // lanes of one group within this warp
+#pragma unroll
+    for (int o = kGroupPairs; o < 32; o <<= 1) {
+        if (o < seg) {                                     // warp-uniform
+            a0 = add3(a0, make_float4(__shfl_xor_sync(0xffffffffu, a0.x, o), __shfl_xor_sync(0xffffffffu, a0.y, o),
+                                      __shfl_xor_sync(0xffffffffu, a0.z, o), 0.f));
+            a1 = add3(a1, make_float4(__shfl_xor_sync(0xffffffffu, a1.x, o), __shfl_xor_sync(0xffffffffu, a1.y, o),
+                                      __shfl_xor_sync(0xffffffffu, a1.z, o), 0.f));
+        }
+    }
+    LIME_WTRACE(1);
+    if (active && sl.s % kWarpSplits == 0) {
+        float4* w = wpart + (static_cast<int64_t>(sl.gslot) * warp_blocks(S2) + sl.s / kWarpSplits) * kGroupTargets;
+        w[2 * sl.p] = a0;
+        w[2 * sl.p + 1] = a1;
+    }
+}
+
+// Target (round slot ct) of the CTA: its warp block sums added as the top of the tree.
+__device__ __forceinline__ float4 small_target_sum(const float4* wpart, int ct, int S2) {
+    const int nb = warp_blocks(S2);
+    const float4* w = wpart + static_cast<int64_t>(ct / kGroupTargets) * nb * kGroupTargets + ct % kGroupTargets;
+    if (nb == 1) return w[0];
+    if (nb == 2) return add3(w[0], w[kGroupTargets]);
+    return add3(add3(w[0], w[kGroupTargets]), add3(w[2 * kGroupTargets], w[3 * kGroupTargets]));
+}
+
+struct SmallArgs {
+    const float4* bodies;
+    int64_t n_src, tgt_begin, tgt_count;
+    float eps2;
+    float4* accel;
+    int S, S2, L, chunk;
+    int64_t groups;
+};
+
+__global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const __grid_constant__ SmallArgs a) {
+    extern __shared__ __align__(128) uint8_t small_smem[];
+    float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
+    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.S, a.L));   // [slots][blocks][4]
+    pdl_enter();
+    const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
+    const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
+    stage_all<false>(src, a.bodies, a.n_src, a.L);
+    __syncthreads();
+    const SmallLane sl(a.S2);
+    const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
+    const int ct = static_cast<int>(threadIdx.x);
+    // rounds of `slots` groups (one round by default); every lane calls small_lane_sum (whole warps
+    // take part in its butterfly), lanes beyond the round's groups inactive
+    for (int64_t r0 = gb; r0 < ge; r0 += slots) {
+        const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
+        small_lane_sum(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
+                       a.S2, a.n_src, a.chunk, a.eps2, wpart);
+        __syncthreads();
+        const int64_t t = r0 * kGroupTargets + ct;
+        if (ct < ng * kGroupTargets && t < a.tgt_count) a.accel[t] = small_target_sum(wpart, ct, a.S2);
+        __syncthreads();                               // wpart[] is reused by the next round
+    }
+}
+
+static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream) {
+    const SmallPlan p = small_plan(f.n_src, f.tgt_count, device_num_sms());
+    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&force_small_kernel), small_smem_bound());
     if (e != cudaSuccess) return e;
-    const int64_t ctas = ceil_div<int64_t>(a.tgt_count, 32);
-    return launch_pdl(&force_small_kernel, dim3(static_cast<unsigned>(ctas)), dim3(32 * ceil_div(a.splits, 2)), smem,
-                      stream, a);
+    SmallArgs a;
+    a.bodies = f.bodies;
+    a.n_src = f.n_src;
+    a.tgt_begin = f.tgt_begin;
+    a.tgt_count = f.tgt_count;
+    a.eps2 = f.eps2;
+    a.accel = f.accel;
+    a.S = p.S;
+    a.S2 = p.S2;
+    a.L = p.L;
+    a.chunk = p.chunk;
+    a.groups = p.groups;
+    return launch_pdl(&force_small_kernel, dim3(static_cast<unsigned>(p.grid)), dim3(static_cast<unsigned>(p.block)),
+                      p.smem, stream, a);
 }
 
 // =====================================================================================
 // Whole simulation in one persistent launch (n <= kSmallMaxSources; the paper's repeated
 // task-graph pass, at its own 4096-body size, Table 3). At this size a
 // step is a few microseconds of FP32 work, so launch gaps and a separate integrator pass cost as
-// much as the forces. One cooperative grid (every CTA resident) runs all `steps`: per step each
-// warp stages its source split from the current position buffer (L2, ld.global.cg), each CTA
-// computes the forces on its 32-target groups exactly as force_small_kernel does, and warp 0
-// applies the integrator (integrate_kernel's arithmetic) and writes the new positions into the
-// other buffer; then a grid barrier. Positions ping-pong between `pos` and a workspace copy; a
-// velocity is only ever touched by its target's thread. Bit-identical to `steps` x
+// much as the forces. One cooperative grid (one CTA per SM, every CTA resident) runs all `steps`
+// with force_small_kernel's decomposition: per step each CTA bulk-copies the current positions
+// into its padded source slots (one mbarrier per split; the copies read what the other CTAs wrote
+// in the previous step, ordered by the grid barrier's release/acquire and a proxy fence), computes
+// its groups' split partials and their tree sums; one thread per target applies the integrator
+// (integrate_kernel's arithmetic) and stores the new position into the other buffer; then a grid
+// barrier. Positions ping-pong between `pos` and a workspace copy. Bit-identical to `steps` x
 // (lime_map_nbody + lime_map_nbody_integrate).
-// (A CTA-pair variant -- clusters of 2, one packed target pair per lane, split partials combined
-// through DSMEM -- was measured slower at 4096: 1024 packed warps leave ~2 per SM sub-partition,
-// too few to hide the dependent FFMA2/MUFU chains; see profiles/experiments.)
 // =====================================================================================
 struct SimArgs {
     float4* pos;        // [n] in/out
@@ -543,9 +702,8 @@ struct SimArgs {
     unsigned* bar;      // [2] grid barrier arrivals, exits (zero between launches)
     int64_t n;
     int32_t steps;
-    int32_t splits;
-    int32_t chunk;
-    int64_t split_len;
+    int32_t S, S2, L, chunk;
+    int64_t groups;
     float eps2, dt;
 };
 
@@ -562,51 +720,44 @@ __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(16 * kMaxSplitsSmall) simulate_small_kernel(const __grid_constant__ SimArgs a) {
+
+__global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(const __grid_constant__ SimArgs a) {
     extern __shared__ __align__(128) uint8_t small_smem[];
-    float4* src = reinterpret_cast<float4*>(small_smem);                                   // [S][split_len]
-    float4* part = reinterpret_cast<float4*>(small_smem + a.splits * a.split_len * 16);   // [S][32]
-    const int warp = threadIdx.x >> 5;                // owns splits 2 warp, 2 warp + 1 (force_small_kernel's map)
-    const unsigned lane = lane_id();
-    const SmallLane sl;
-    const int64_t groups = ceil_div<int64_t>(a.n, 32);
-    const int64_t w0 = static_cast<int64_t>(2 * warp) * a.split_len;
-    const int wlen = static_cast<int>(mn<int64_t>(a.n, w0 + 2 * a.split_len) - w0);
-    const int64_t j0 = static_cast<int64_t>(sl.split) * a.split_len;
-    const int len = sl.split < a.splits ? static_cast<int>(mn<int64_t>(a.n, j0 + a.split_len) - j0) : 0;
+    float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
+    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.S, a.L));   // [slots][blocks][4]
+    const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
+    const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
+    const SmallLane sl(a.S2);
+    const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
+    const int ct = static_cast<int>(threadIdx.x);      // combine thread: one target of the round's groups
     unsigned barrier_target = 0;
 
     for (int32_t k = 0; k < a.steps; ++k) {
         const float4* cur = (k & 1) ? a.pos_alt : a.pos;
         float4* nxt = (k & 1) ? a.pos : a.pos_alt;
-        for (int j = static_cast<int>(lane); j < wlen; j += 32) src[w0 + j] = __ldcg(cur + w0 + j);
-        __syncwarp();
-        for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
-            const int64_t t = g * 32 + lane;
-            const bool valid = t < a.n;
-            const float4 p = __ldcg(cur + (valid ? t : a.n - 1));
-            Interact<2, true> it;
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int64_t tr = g * 32 + 2 * sl.q + r;
-                it.set(r, __ldcg(cur + (tr < a.n ? tr : a.n - 1)));
-            }
-            it.zero_all();
-            split_sum(it, src + j0, len, a.chunk, a.eps2);
-            if (sl.split < a.splits) {
-                part[sl.split * 32 + 2 * sl.q] = it.result(0);
-                part[sl.split * 32 + 2 * sl.q + 1] = it.result(1);
-            }
+        LIME_TRACE_AT(k, 0);
+#ifdef LIME_TRACE
+        if (blockIdx.x == 0 && threadIdx.x == 0) g_lime_step = k;
+        __syncthreads();
+#endif
+        LIME_TRACE_AT(k, 5);
+        stage_all<true>(src, cur, a.n, a.L);       // what every CTA wrote in the previous step (L2)
+        __syncthreads();
+        LIME_TRACE_AT(k, 6);
+        for (int64_t r0 = gb; r0 < ge; r0 += slots) {
+            const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
+            const int64_t t = r0 * kGroupTargets + ct;
+            const bool owner = ct < ng * kGroupTargets && t < a.n;
+            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (owner) v = a.vel[t];                   // issued before the force work: latency hidden
+            small_lane_sum(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
+                           a.eps2, wpart);
+            LIME_TRACE_AT(k, 4);
             __syncthreads();
-            if (warp == 0 && valid) {
-                float4 acc = part[lane];
-#pragma unroll 8
-                for (int s = 1; s < a.splits; ++s) {
-                    const float4 q = part[s * 32 + lane];
-                    acc.x += q.x; acc.y += q.y; acc.z += q.z;
-                }
-                float4 v = a.vel[t];
-                float4 pn = p;
+            LIME_TRACE_AT(k, 1);
+            if (owner) {
+                const float4 acc = small_target_sum(wpart, ct, a.S2);
+                float4 pn = src[padded(static_cast<int>(t), a.L)];
                 v.x = fmaf(acc.x, a.dt, v.x);
                 v.y = fmaf(acc.y, a.dt, v.y);
                 v.z = fmaf(acc.z, a.dt, v.z);
@@ -616,19 +767,19 @@ __global__ void __launch_bounds__(16 * kMaxSplitsSmall) simulate_small_kernel(co
                 a.vel[t] = v;
                 __stcg(nxt + t, pn);
             }
-            __syncthreads();                       // part[] is reused by the next group
+            __syncthreads();                           // wpart[] is reused by the next round
         }
+        LIME_TRACE_AT(k, 2);
         const bool last = (k + 1 == a.steps);
         if (!last || (a.steps & 1)) {
             barrier_target += gridDim.x;
             grid_barrier(a.bar, barrier_target);
         }
+        LIME_TRACE_AT(k, 3);
     }
-    if ((a.steps & 1) && warp == 0) {              // final positions are in pos_alt: copy own targets back
-        for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
-            const int64_t t = g * 32 + lane;
-            if (t < a.n) a.pos[t] = __ldcg(a.pos_alt + t);
-        }
+    if (a.steps & 1) {                                 // the last step wrote pos_alt; every CTA is past its reads
+        for (int64_t t = gb * kGroupTargets + ct; t < mn<int64_t>(a.n, ge * kGroupTargets); t += blockDim.x)
+            a.pos[t] = __ldcg(a.pos_alt + t);
     }
     if (threadIdx.x == 0) {                        // the last CTA out leaves the barrier zeroed
         __threadfence();
@@ -638,6 +789,15 @@ __global__ void __launch_bounds__(16 * kMaxSplitsSmall) simulate_small_kernel(co
         }
     }
 }
+
+#ifdef LIME_TRACE
+extern "C" int lime_debug_trace(void* host, size_t bytes) {
+    return static_cast<int>(cudaMemcpyFromSymbol(host, g_lime_trace, mn(bytes, sizeof(g_lime_trace))));
+}
+extern "C" int lime_debug_wtrace(void* host, size_t bytes) {
+    return static_cast<int>(cudaMemcpyFromSymbol(host, g_lime_wtrace, mn(bytes, sizeof(g_lime_wtrace))));
+}
+#endif
 
 // workspace: [grid barrier, 256 B][force workspace (its tickets first)][pos_alt / accel, n x 16 B] --
 // every zero-invariant word sits at an offset that does not depend on n, so a workspace reused
@@ -659,6 +819,14 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
         }
         return cudaSuccess;
     }
+    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&simulate_small_kernel), small_smem_bound());
+    if (e != cudaSuccess) return e;
+    int max_grid = device_num_sms();
+    const LaunchOverride& ov = launch_override();
+    if (ov.grid_ctas > 0) max_grid = mn(max_grid, ov.grid_ctas);
+    const SmallPlan p = small_plan(n, n, max_grid);
+    const int occ = cached_occupancy(reinterpret_cast<const void*>(&simulate_small_kernel), p.block, p.smem);
+    if (occ < 1) return cudaErrorInvalidConfiguration;          // one CTA per SM is all the grid needs
     SimArgs a;
     a.pos = pos;
     a.vel = vel;
@@ -666,26 +834,17 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.bar = reinterpret_cast<unsigned*>(w);
     a.n = n;
     a.steps = steps;
-    a.splits = splits(n);
-    a.chunk = chunk_len(n);
-    a.split_len = chunks_per_split(n) * a.chunk;
+    a.S = p.S;
+    a.S2 = p.S2;
+    a.L = p.L;
+    a.chunk = p.chunk;
+    a.groups = p.groups;
     a.eps2 = eps2;
     a.dt = dt;
-    const int block = 32 * ceil_div(a.splits, 2);
-    const size_t smem = static_cast<size_t>(a.splits) * a.split_len * 16 + static_cast<size_t>(a.splits) * 32 * 16;
-    cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&simulate_small_kernel),
-                                        static_cast<int>(kSmallMaxSources * 16 + kMaxSplitsSmall * 32 * 16));
-    if (e != cudaSuccess) return e;
-    const int occ = cached_occupancy(reinterpret_cast<const void*>(&simulate_small_kernel), block, smem);
-    if (occ < 1) return cudaErrorInvalidConfiguration;
-    const int64_t groups = ceil_div<int64_t>(n, 32);
-    int grid = static_cast<int>(mn<int64_t>(groups, static_cast<int64_t>(occ) * device_num_sms()));
-    const LaunchOverride& ov = launch_override();
-    if (ov.grid_ctas > 0) grid = static_cast<int>(mn<int64_t>(grid, ov.grid_ctas));
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(static_cast<unsigned>(grid));
-    cfg.blockDim = dim3(static_cast<unsigned>(block));
-    cfg.dynamicSmemBytes = smem;
+    cfg.gridDim = dim3(static_cast<unsigned>(p.grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(p.block));
+    cfg.dynamicSmemBytes = p.smem;
     cfg.stream = stream;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeCooperative;         // all CTAs co-resident (the grid barrier needs it)
@@ -845,6 +1004,7 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.splits = splits(n_src);
     a.chunk = chunk_len(n_src);
     a.split_len = chunks_per_split(n_src) * a.chunk;
+    a.tree = n_src <= kSmallMaxSources;
     a.counters = static_cast<unsigned*>(ws);
     a.uniform = nullptr;
     a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count) + flags_bytes(n_src));
