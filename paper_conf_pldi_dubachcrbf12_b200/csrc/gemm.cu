@@ -482,6 +482,224 @@ gemm2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__
     }
 }
 
+// =====================================================================================
+// Wide pair tile (round 2): a CTA pair computes 256 x 512 of C as two N = 256 halves H0 | H1 that
+// fill each SM's 512 TMEM columns. Per 64-element K slice each CTA stages 128 rows of A and 2 x 128
+// rows of Bt (48 KB), so a call moves 3/4 of the 256 x 256 tile's L2->SM bytes (8192^3: 6.4 vs
+// 8.6 GB -- what cuBLAS moves; the kernel is power-capped, so fewer bytes buy clock).
+// With no spare TMEM for a second accumulator, the tile boundary is overlapped instead:
+//  * 8 epilogue warps (two per TMEM lane quadrant, 128 columns each) pull a half into registers
+//    (4 x tcgen05.ld.32x32b.x32, one wait) and release it at once; the global stores (TMA, one
+//    32 x 32 smem box per warp) follow from registers while the next tile's MMAs run;
+//  * the MMA thread starts tile t+1 on H0 as soon as H0 is released and defers the H1 MMAs of
+//    the first STAGES - 1 K slices (their smem stages stay held) until H1 is released too.
+// =====================================================================================
+namespace wide {
+constexpr int BM = 128;                   // rows of A per CTA (pair tile: 256)
+constexpr int BN = 512;                   // pair tile N: two N = 256 MMAs per K step
+constexpr int STAGES = 4;
+constexpr int kThreads = 320;             // producer, MMA, 8 epilogue warps
+constexpr uint32_t kStageA = BM * BK * 2;             // 16 KB
+constexpr uint32_t kStageBh = 128 * BK * 2;           // 16 KB per half (this CTA's 128 rows of an N = 256 chunk)
+constexpr uint32_t kStageBytes = kStageA + 2 * kStageBh;
+constexpr uint32_t kEpiBox = 32 * 32 * 4;             // one 32 x 32 fp32 box per epilogue warp
+constexpr uint32_t kEpiBytes = 8 * kEpiBox;
+constexpr size_t kSmemBytes = 1024 + STAGES * kStageBytes + kEpiBytes + 256;
+constexpr int kDefer = STAGES - 1;
+constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (static_cast<uint32_t>(256 >> 3) << 17) |
+                            (static_cast<uint32_t>(256 >> 4) << 24);
+}  // namespace wide
+
+// 4 x 32 consecutive fp32 columns of this warp's TMEM lane quadrant, one wait
+__device__ __forceinline__ void tmem_ld128(uint32_t taddr, uint32_t (&r)[128]) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+            "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+            : "=r"(r[32 * q + 0]), "=r"(r[32 * q + 1]), "=r"(r[32 * q + 2]), "=r"(r[32 * q + 3]), "=r"(r[32 * q + 4]),
+              "=r"(r[32 * q + 5]), "=r"(r[32 * q + 6]), "=r"(r[32 * q + 7]), "=r"(r[32 * q + 8]), "=r"(r[32 * q + 9]),
+              "=r"(r[32 * q + 10]), "=r"(r[32 * q + 11]), "=r"(r[32 * q + 12]), "=r"(r[32 * q + 13]),
+              "=r"(r[32 * q + 14]), "=r"(r[32 * q + 15]), "=r"(r[32 * q + 16]), "=r"(r[32 * q + 17]),
+              "=r"(r[32 * q + 18]), "=r"(r[32 * q + 19]), "=r"(r[32 * q + 20]), "=r"(r[32 * q + 21]),
+              "=r"(r[32 * q + 22]), "=r"(r[32 * q + 23]), "=r"(r[32 * q + 24]), "=r"(r[32 * q + 25]),
+              "=r"(r[32 * q + 26]), "=r"(r[32 * q + 27]), "=r"(r[32 * q + 28]), "=r"(r[32 * q + 29]),
+              "=r"(r[32 * q + 30]), "=r"(r[32 * q + 31])
+            : "r"(taddr + static_cast<uint32_t>(32 * q)));
+    }
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(wide::kThreads, 1)
+gemm_wide_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+                 const __grid_constant__ CUtensorMap tmap_c, const __grid_constant__ Params2 p) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* epi = smem + wide::STAGES * wide::kStageBytes;
+    uint64_t* full = reinterpret_cast<uint64_t*>(epi + wide::kEpiBytes);
+    uint64_t* empty = full + wide::STAGES;
+    uint64_t* tfull = empty + wide::STAGES;
+    uint64_t* tempty = tfull + 1;                      // [2]: H0, H1 released
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+    const bool leader = (rank == 0);
+    const int cluster = blockIdx.x >> 1;
+    const int nclusters = gridDim.x >> 1;
+
+    if (warp == 0 && lane == 0) {
+        prefetch_tmap(&tmap_a);
+        prefetch_tmap(&tmap_b);
+        prefetch_tmap(&tmap_c);
+        for (int s = 0; s < wide::STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        mbar_init(&tfull[0], 1);
+        mbar_init(&tempty[0], 16);       // 8 epilogue warps x 2 CTAs (the leader's copy is the one used)
+        mbar_init(&tempty[1], 16);
+        fence_mbar_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_addr(tmem_slot)), "r"(kTmemCols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    }
+    tc_fence_before();
+    cluster_sync();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int t = cluster; t < p.num_tiles; t += nclusters) {
+                int mb, nb;
+                tile_coords2(t, p, mb, nb);
+                const int arow = mb * 256 + static_cast<int>(rank) * wide::BM;
+                const int brow = nb * wide::BN + static_cast<int>(rank) * 128;
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&empty[s], ph ^ 1);
+                    uint8_t* sa = smem + s * wide::kStageBytes;
+                    const uint32_t lbar = mapa_shared(smem_addr(&full[s]), 0);
+                    if (leader) mbar_arrive_expect_tx(&full[s], 2 * wide::kStageBytes);
+                    tma_load_2d_pair(&tmap_a, sa, lbar, kb * BK, arow);
+                    tma_load_2d_pair(&tmap_b, sa + wide::kStageA, lbar, kb * BK, brow);
+                    tma_load_2d_pair(&tmap_b, sa + wide::kStageA + wide::kStageBh, lbar, kb * BK, brow + 256);
+                    if (++s == wide::STAGES) { s = 0; ph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (leader && lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            int local = 0;
+            auto mma_half = [&](int st, int kb, int h) {
+                const uint32_t sa = smem_addr(smem + st * wide::kStageBytes);
+                const uint32_t sb = sa + wide::kStageA + static_cast<uint32_t>(h) * wide::kStageBh;
+#pragma unroll
+                for (int k = 0; k < BK / UMMA_K; ++k)
+                    tc_mma_pair(tmem_base + static_cast<uint32_t>(h * 256), smem_desc_sw128(sa + k * UMMA_K * 2),
+                                smem_desc_sw128(sb + k * UMMA_K * 2), wide::kIdesc, (kb | k) != 0);
+            };
+            for (int t = cluster; t < p.num_tiles; t += nclusters, ++local) {
+                const uint32_t par = static_cast<uint32_t>(local & 1) ^ 1u;
+                mbar_wait(&tempty[0], par);                // H0 drained (previous tile)
+                tc_fence_after();
+                int dst[wide::kDefer], dkb[wide::kDefer], nd = 0;
+                bool h1_free = false;
+                for (int kb = 0; kb < p.num_k; ++kb) {
+                    mbar_wait(&full[s], ph);
+                    tc_fence_after();
+                    mma_half(s, kb, 0);
+                    if (!h1_free && nd < wide::kDefer) {   // H1 still draining: hold this stage
+                        dst[nd] = s;
+                        dkb[nd] = kb;
+                        ++nd;
+                    } else {
+                        if (!h1_free) {
+                            mbar_wait(&tempty[1], par);
+                            tc_fence_after();
+                            h1_free = true;
+                            for (int d = 0; d < nd; ++d) {
+                                mma_half(dst[d], dkb[d], 1);
+                                tc_commit_pair(&empty[dst[d]]);
+                            }
+                            nd = 0;
+                        }
+                        mma_half(s, kb, 1);
+                        tc_commit_pair(&empty[s]);
+                    }
+                    if (++s == wide::STAGES) { s = 0; ph ^= 1; }
+                }
+                if (!h1_free) {                            // num_k <= kDefer
+                    mbar_wait(&tempty[1], par);
+                    tc_fence_after();
+                    for (int d = 0; d < nd; ++d) {
+                        mma_half(dst[d], dkb[d], 1);
+                        tc_commit_pair(&empty[dst[d]]);
+                    }
+                }
+                tc_commit_pair(&tfull[0]);
+            }
+        }
+        __syncwarp();
+    } else {
+        // ----------------------------------------------------------- epilogue (warps 2..9)
+        const int quad = warp & 3;
+        const int colpart = (warp - 2) >> 2;               // 128-column part of each half
+        const uint32_t tempty_leader = mapa_shared(smem_addr(&tempty[0]), 0);
+        const uint32_t box = smem_addr(epi + (warp - 2) * wide::kEpiBox);
+        int local = 0;
+        for (int t = cluster; t < p.num_tiles; t += nclusters, ++local) {
+            int mb, nb;
+            tile_coords2(t, p, mb, nb);
+            mbar_wait(&tfull[0], static_cast<uint32_t>(local & 1));
+            tc_fence_after();
+            const int row0 = mb * 256 + static_cast<int>(rank) * wide::BM + quad * 32;
+#pragma unroll 1
+            for (int h = 0; h < 2; ++h) {
+                uint32_t r[128];
+                tmem_ld128(tmem_base + (static_cast<uint32_t>(quad * 32) << 16) +
+                               static_cast<uint32_t>(h * 256 + colpart * 128), r);
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cluster(tempty_leader + static_cast<uint32_t>(h * 8));
+#pragma unroll
+                for (int b = 0; b < 4; ++b) {
+                    if (lane == 0) bulk_wait_read<0>();    // the previous store has read the box
+                    __syncwarp();
+#pragma unroll
+                    for (int q = 0; q < 8; ++q)
+                        st_shared_f4(box + static_cast<uint32_t>(lane * 128 + ((q ^ (lane & 7)) << 4)),
+                                     __uint_as_float(r[32 * b + 4 * q]), __uint_as_float(r[32 * b + 4 * q + 1]),
+                                     __uint_as_float(r[32 * b + 4 * q + 2]), __uint_as_float(r[32 * b + 4 * q + 3]));
+                    fence_proxy_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        tma_store_2d(&tmap_c, epi + (box - smem_addr(epi)), nb * wide::BN + h * 256 + colpart * 128 + b * 32,
+                                     row0);
+                        bulk_commit();
+                    }
+                }
+            }
+        }
+        if (lane == 0) bulk_wait_all();
+    }
+
+    tc_fence_before();
+    cluster_sync();
+    if (warp == 1) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(tmem_base), "r"(kTmemCols) : "memory");
+    }
+}
+
 // ------------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -522,8 +740,34 @@ static bool make_map_c(CUtensorMap* map, void* base, uint64_t rows, uint64_t col
 cudaError_t launch_bf16(const uint16_t* A, const uint16_t* Bt, float* C, int64_t M, int64_t N, int64_t K,
                         cudaStream_t stream) {
     const LaunchOverride& ov = launch_override();
-    const bool pair = ov.per_thread == 2 || (ov.per_thread != 1 && M >= 256);
+    // per_thread override: 1 = 1-CTA kernel, 2 = 256 x 256 pair tile, 3 = the same with direct
+    // stores, 4 = 256 x 512 pair tile; default: wide tile when it fits, else 256 x 256.
+    const bool c_tma_ok = (N & 3) == 0 && (reinterpret_cast<uintptr_t>(C) & 15) == 0;
+    const bool wide_tile = ov.per_thread == 4 || (ov.per_thread == 0 && M >= 256 && N >= 512 && c_tma_ok);
+    const bool pair = ov.per_thread == 2 || ov.per_thread == 3 || (ov.per_thread == 0 && M >= 256);
     CUtensorMap ma, mb;
+    if (wide_tile) {
+        CUtensorMap mc;
+        if (!c_tma_ok || !make_map(&ma, A, M, K, wide::BM) || !make_map(&mb, Bt, N, K, 128) || !make_map_c(&mc, C, M, N))
+            return cudaErrorInvalidValue;
+        Params2 p;
+        p.C = C;
+        p.tma_store = 1;
+        p.M = static_cast<int>(M);
+        p.N = static_cast<int>(N);
+        p.K = static_cast<int>(K);
+        p.num_m = static_cast<int>(ceil_div<int64_t>(M, 256));
+        p.num_n = static_cast<int>(ceil_div<int64_t>(N, wide::BN));
+        p.num_k = static_cast<int>(ceil_div<int64_t>(K, BK));
+        p.num_tiles = p.num_m * p.num_n;
+        p.group = ov.block_threads > 0 ? ov.block_threads : 8;   // override: raster group (sweep)
+        cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&gemm_wide_kernel), static_cast<int>(wide::kSmemBytes));
+        if (e != cudaSuccess) return e;
+        int clusters = ov.grid_ctas > 0 ? mx(1, ov.grid_ctas / 2) : device_num_sms() / 2;
+        clusters = mn(clusters, p.num_tiles);
+        gemm_wide_kernel<<<2 * clusters, wide::kThreads, wide::kSmemBytes, stream>>>(ma, mb, mc, p);
+        return cudaGetLastError();
+    }
     if (pair) {
         if (!make_map(&ma, A, M, K, two::BM) || !make_map(&mb, Bt, N, K, two::BN / 2)) return cudaErrorInvalidValue;
         Params2 p;

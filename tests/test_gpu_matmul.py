@@ -84,3 +84,24 @@ def test_matmul_epilogue_forms_identical(lime, M, N, K):
     assert torch.equal(C_tma, C_st)
     e, fro = _check(C_tma.cpu().numpy(), A, Bt)
     assert e <= MATMUL_RTOL and fro <= MATMUL_RTOL
+
+
+@pytest.mark.parametrize("M,N,K", [(256, 512, 64), (300, 520, 136), (513, 1028, 200), (1024, 1536, 512),
+                                   (257, 4100, 8)])
+def test_matmul_tile_kernels_identical(lime, M, N, K):
+    # 1-CTA 128x256, pair 256x256 (TMA-store and direct epilogues) and the wide 256x512 pair tile
+    # (default for M >= 256, N >= 512) add every dot product in the same K order -> the same bits;
+    # K <= 192 exercises the wide tile's deferred-H1 path with fewer K slices than held stages,
+    # grid_ctas=2 (one pair doing every tile) its accumulator-release parity across many tiles
+    A, Bt = inputs.matmul_operands(M, N, K, seed=M + 5 * N + K)
+    C_def = lime.map_matmul_bf16(_bf(A), _bf(Bt))
+    for pt in (1, 2, 3, 4):
+        with lime.launch_override(per_thread=pt):
+            assert torch.equal(lime.map_matmul_bf16(_bf(A), _bf(Bt)), C_def), pt
+    with lime.launch_override(per_thread=4, grid_ctas=2):
+        assert torch.equal(lime.map_matmul_bf16(_bf(A), _bf(Bt)), C_def)
+    for g in (1, 3, 16):
+        with lime.launch_override(per_thread=4, block_threads=g):
+            assert torch.equal(lime.map_matmul_bf16(_bf(A), _bf(Bt)), C_def), g
+    e, fro = _check(C_def.cpu().numpy(), A, Bt)
+    assert e <= MATMUL_RTOL and fro <= MATMUL_RTOL

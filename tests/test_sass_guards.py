@@ -54,7 +54,7 @@ def test_nbody_uses_packed_fp32_and_mufu_and_bulk_copy(sass):
 
 
 def test_gemm_is_tcgen05(sass):
-    for pat in (r"gemm_kernel", r"gemm2_kernel"):
+    for pat in (r"gemm_kernel", r"gemm2_kernel", r"gemm_wide_kernel"):
         ops = " ".join(_fn(sass, pat))
         assert "UTCHMMA" in ops or "UTCQMMA" in ops   # tcgen05.mma
         assert "UTMALDG" in ops                        # TMA tensor loads
@@ -62,10 +62,11 @@ def test_gemm_is_tcgen05(sass):
         assert "HMMA" not in ops.replace("UTCHMMA", "")
 
 
-def test_gemm2_is_two_cta_tcgen05_with_tma_store(sass):
-    # the production kernel: cta_group::2 MMAs, pair-wide TMA loads, the
-    # TMA-store epilogue and tcgen05.ld
-    ops = " ".join(_fn(sass, r"gemm2_kernel"))
+@pytest.mark.parametrize("kernel", [r"gemm2_kernel", r"gemm_wide_kernel"])
+def test_pair_gemms_are_two_cta_tcgen05_with_tma_store(sass, kernel):
+    # the production kernels (gemm_wide_kernel is the default for M >= 256,
+    # N >= 512 since round 2): cta_group::2 MMAs, pair-wide TMA loads, TMA-store epilogue, tcgen05.ld
+    ops = " ".join(_fn(sass, kernel))
     assert "UTCHMMA.2CTA" in ops
     assert "UTMALDG" in ops
     assert "UTMASTG" in ops
