@@ -47,6 +47,7 @@ FP32_LANE_OPS_PER_INTERACTION = 12  # 3 FADD + 3 FFMA (r^2) + 3 FMUL + 3 FFMA (a
 FP32_LANE_OPS_UNIFORM_MASS = 11
 SM_MAX_MHZ_NOMINAL = 1965.0
 SMS_B200 = 148
+IDEA_SASS_PER_UNIT = 663           # idea_kernel loop: SASS instructions per 16-byte unit (2 blocks)
 
 
 # ----------------------------------------------------------------------------- peaks
@@ -579,15 +580,22 @@ def run_extras(peaks, flush):
     ek, _ = lime.idea_key_schedule(inputs.crypt_key())
     enc = torch.empty_like(data)
     med, _ = time_launches(lambda: lime.map_idea(data, ek, out=enc), 30, 3, flush)
-    gbs = 2.0 * data.numel() / (med * 1e-3) / 1e9
+    # integer-issue roofline: the IDEA round function is multiplications mod
+    # 2^16+1, additions and XORs on the ALU/FMA(IMAD) pipes; the bound is instruction issue, one
+    # warp-instruction per SMSP per clock = 148 x 4 x 32 thread-instructions/clk. The kernel's
+    # loop runs IDEA_SASS_PER_UNIT SASS instructions per 16-byte unit (two 8-byte blocks; counted
+    # from cuobjdump, pinned by tests/test_sass_guards.py).
+    units = data.numel() / 16.0
+    issue_peak = SMS_B200 * 4 * 32 * SM_MAX_MHZ_NOMINAL * 1e6
+    ach = units * IDEA_SASS_PER_UNIT / (med * 1e-3)
     out["jg_crypt"] = {"workload": "F4: JG-Crypt IDEA-ECB over 3 MiB (Table 3)", "value": data.numel() / (med * 1e-3),
-                       "unit": "bytes/s", "ms_per_launch": med,
-                       "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm,
-                                    "traffic": None,
-                                    "note": "not HBM-bound at 3 MiB (6 MB of traffic = 1 us at HBM speed): integer-issue-bound "
-                                            "(ncu r01n: issue active 78 %; 333 SASS instructions per 8-byte block, 34 "
-                                            "multiplications mod 2^16+1), one wave of 768 CTAs; ~6 us of the event-timed "
-                                            "launch is the launch floor (tools/launch_floor.py)"}}
+                       "unit": "bytes/s", "ms_per_launch": med, "hbm_GBs": 2.0 * data.numel() / (med * 1e-3) / 1e9,
+                       "roofline": {"bound": "issue", "achieved": ach / 1e12, "peak": issue_peak / 1e12,
+                                    "unit": "T thread-instructions/s", "frac": ach / issue_peak, "traffic": None,
+                                    "sass_per_16B_unit": IDEA_SASS_PER_UNIT,
+                                    "note": "one wave of CTAs over 3 MiB: the issue-bound work is ~3.5 us at 1965 MHz, so "
+                                            "launch/ramp (~5-6 us of the event-timed launch, tools/launch_floor.py) "
+                                            "dominates; HBM traffic (6 MB) is 1 us at HBM speed"}}
     del data, enc
 
     # reduction `!`: sum over 2^28 fp32 (1 GiB)

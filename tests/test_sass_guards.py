@@ -71,3 +71,27 @@ def test_pair_gemms_are_two_cta_tcgen05_with_tma_store(sass, kernel):
     assert "UTMALDG" in ops
     assert "UTMASTG" in ops
     assert "LDTM" in ops
+
+
+def test_idea_loop_instruction_count_matches_bench(sass):
+    # bench.py's JG-Crypt issue roofline divides by IDEA_SASS_PER_UNIT: the grid-stride loop body
+    # (one 16-byte unit = two IDEA blocks) must still be that long (+-3 %)
+    import re
+    import bench
+    lib = lime_build.build()
+    out = subprocess.run(["cuobjdump", "-sass", lib], capture_output=True, text=True, check=True).stdout
+    lines, cur = [], False
+    for line in out.splitlines():
+        m = re.search(r"Function : (\S+)", line)
+        if m:
+            cur = "idea_kernel" in m.group(1)
+        elif cur:
+            lines.append(line)
+    addr = [int(m.group(1), 16) for ln in lines for m in [re.search(r"/\*([0-9a-f]{4})\*/", ln)] if m]
+    back = [(int(m.group(2), 16), int(m.group(1), 16)) for ln in lines
+            for m in [re.search(r"/\*([0-9a-f]{4})\*/\s+@!?P\d\s+BRA\s+0x([0-9a-f]+)", ln)] if m]
+    loops = [(dst, src) for dst, src in back if dst < src]
+    assert loops and addr
+    dst, src = max(loops, key=lambda x: x[1] - x[0])
+    n = (src - dst) // 16 + 1
+    assert abs(n - bench.IDEA_SASS_PER_UNIT) <= 0.03 * bench.IDEA_SASS_PER_UNIT, n
