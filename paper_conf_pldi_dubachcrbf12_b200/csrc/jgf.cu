@@ -33,6 +33,8 @@ namespace jgf {
 constexpr int kSeriesM = 1000;            // JGF: TrapezoidIntegrate(0, 2, 1000, ...)
 constexpr int kSeriesNodes = 1024;        // m + 1 = 1001 nodes, zero-padded
 constexpr int kSeriesBlock = 128;
+constexpr int kSeriesPadded = kSeriesM + kSeriesM / 8 + 1;   // smem table slots (one pad per 8)
+__device__ __forceinline__ int series_pos(int p) { return p + (p >> 3); }
 
 // Node weights g_i = w_i (x_i + 1)^{x_i} (w = 1/2 at the ends, 0 at the skipped node x_{m-1}), rounded
 // to T, as a kernel parameter: the kernel reads them with compile-time offsets, so they arrive through
@@ -135,10 +137,17 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
                                                               int64_t n0, int64_t count, T* __restrict__ out) {
     using T2 = typename Vec2<T>::type;
     constexpr int NU = kSeriesNodes / R;
-    __shared__ T sc[kSeriesM], ss[kSeriesM];
+    // Table entry p sits at p + p/8: the lanes of a warp gather p = (R n u) mod m for consecutive n,
+    // i.e. at a stride of 16u (R = 16), which on the plain layout put most of a warp in one or two
+    // banks (ncu r02: 1.57M excess wavefronts per gather instruction, 3.27M conflicts per launch);
+    // one pad word per 8 entries spreads the strides -- simulated 8.85 -> 2.07 wavefronts per
+    // 32-lane gather, measured 0.52M conflicts. (The launch time did not move: the kernel is
+    // latency-bound, one wave of 5.3 warps per SMSP at ~48 % issue; a 2/4/8-way split of each
+    // coefficient over threads with the u loop unrolled spilled at 64 registers and ran 2-6x slower.)
+    __shared__ T sc[kSeriesPadded], ss[kSeriesPadded];
     const T* gc = series_cos<T>();
     const T* gs = series_sin<T>();
-    for (int i = threadIdx.x; i < kSeriesM; i += blockDim.x) { sc[i] = gc[i]; ss[i] = gs[i]; }
+    for (int i = threadIdx.x; i < kSeriesM; i += blockDim.x) { sc[series_pos(i)] = gc[i]; ss[series_pos(i)] = gs[i]; }
     __syncthreads();
     const T dx = static_cast<T>(2.0 / kSeriesM);
     for (int64_t k = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; k < count;
@@ -149,8 +158,8 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
         int p = 0;
 #pragma unroll
         for (int v = 0; v < R; ++v) {
-            V[v].x = sc[p];
-            V[v].y = ss[p];
+            V[v].x = sc[series_pos(p)];
+            V[v].y = ss[series_pos(p)];
             p += step;
             p -= (p >= kSeriesM) ? kSeriesM : 0;
         }
@@ -174,7 +183,7 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
 #pragma unroll
                 for (int v = 0; v < R; ++v) gn[v] = G.g[un * R + v];
             }
-            const T ur = sc[q], ui = ss[q];
+            const T ur = sc[series_pos(q)], ui = ss[series_pos(q)];
             q += step_u;
             q -= (q >= kSeriesM) ? kSeriesM : 0;
             T2 w0, w1;                                // W_u, even and odd v (two dependency chains)
