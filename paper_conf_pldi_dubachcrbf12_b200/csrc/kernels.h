@@ -15,6 +15,7 @@ struct LaunchOverride {
 const LaunchOverride& launch_override();
 int nbody_variant();   // staging ablation selector (0 = production kernels), see lime_set_nbody_variant
 int device_num_sms();
+void* tensor_map_encoder();   // PFN_cuTensorMapEncodeTiled (gemm.cu), or null
 
 // ------------------------------------------------------------------ N-Body
 namespace nbody {

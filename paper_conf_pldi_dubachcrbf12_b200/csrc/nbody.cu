@@ -19,7 +19,11 @@
 //  * A8 (split-j): S = splits(n_src) source ranges are processed by separate CTAs; the last
 //    CTA of a target tile to finish (atomic ticket) adds the S partials in s order --
 //    one launch, deterministic, self-resetting counters.
+#include <cstring>
 #include <type_traits>
+
+#include <cuda.h>
+#include <cudaTypedefs.h>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -490,8 +494,47 @@ __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int
     }
 }
 
+// TMA staging (n_src % 64 == 0 with 64-body splits, e.g. the paper's 4096 bodies): the sources are
+// a 2-D tensor of 8-byte elements, one row per split ([S][2L]); one box of kStageRows rows x (2L + 2)
+// columns -- the last two columns are out of bounds and zero-filled -- lands in shared memory with
+// a row pitch of (L + 1) float4, i.e. directly in the padded layout. One copy (and mbarrier) per
+// 16 splits = one warp block, so a warp starts as soon as its quarter of the sources has landed
+// (tools/load_mb.cu: 4 x 16-KB copies into all 148 SMs complete in ~1.1k cycles).
+constexpr int kStageRows = 16;
+constexpr int kMaxStageCopies = kMaxSplitsSmall / kStageRows;
+__device__ __forceinline__ void tma_rows(const CUtensorMap* map, void* dst, uint64_t* bar, int row0) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+        :: "r"(smem_addr(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(0), "r"(row0), "r"(smem_addr(bar))
+        : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__host__ __device__ __forceinline__ uint32_t stage_copy_bytes(int L) { return static_cast<uint32_t>(kStageRows * (L + 1) * 16); }
+// threads c < copies: arm copy c's barrier and issue it
+__device__ __forceinline__ void stage_tma(float4* src, const CUtensorMap* map, int S, int L, uint64_t* tbar) {
+    const int c = static_cast<int>(threadIdx.x);
+    if (c < ceil_div(S, kStageRows)) {
+        mbar_arrive_expect_tx(&tbar[c], stage_copy_bytes(L));
+        tma_rows(map, src + static_cast<int64_t>(c) * kStageRows * (L + 1), &tbar[c], c * kStageRows);
+    }
+}
+static bool make_rows_map(CUtensorMap* map, const float4* base, int S, int L) {
+    auto fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(tensor_map_encoder());
+    if (!fn || 2 * L + 2 > 256) return false;
+    const cuuint64_t dims[2] = {static_cast<cuuint64_t>(2 * L), static_cast<cuuint64_t>(S)};
+    const cuuint64_t strides[1] = {static_cast<cuuint64_t>(16 * L)};
+    const cuuint32_t box[2] = {static_cast<cuuint32_t>(2 * L + 2), static_cast<cuuint32_t>(kStageRows)};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, const_cast<float4*>(base), dims, strides, box, estr,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+static bool small_tma_ok(int64_t n_src, int L) { return L == 64 && n_src % L == 0 && tensor_map_encoder() != nullptr; }
+
 struct SmallPlan {
     int S, S2;           // splits(n_src), next_pow2(S)
+    int rows;            // staged source rows (splits; whole 16-row TMA boxes when tma)
+    int tma;
     int L;               // split length (bodies)
     int chunk;
     int64_t groups;      // ceil(targets / 4)
@@ -511,10 +554,12 @@ static SmallPlan small_plan(int64_t n_src, int64_t targets, int max_grid) {
     p.chunk = chunk_len(n_src);
     p.L = static_cast<int>(chunks_per_split(n_src) * p.chunk);
     p.groups = ceil_div<int64_t>(targets, kGroupTargets);
+    p.tma = small_tma_ok(n_src, p.L) ? 1 : 0;
+    p.rows = p.tma ? ceil_div(p.S, kStageRows) * kStageRows : p.S;
     p.grid = static_cast<int>(mx<int64_t>(1, mn<int64_t>(p.groups, max_grid)));
     p.slots = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(p.groups, p.grid), kSmallMaxThreads / (kGroupPairs * p.S2)));
     p.block = ceil_div(p.slots * kGroupPairs * p.S2, 32) * 32;
-    p.smem = small_src_bytes(p.S, p.L) + static_cast<size_t>(p.slots) * warp_blocks(p.S2) * kGroupTargets * 16;
+    p.smem = small_src_bytes(p.rows, p.L) + static_cast<size_t>(p.slots) * warp_blocks(p.S2) * kGroupTargets * 16;
     // One CTA per SM: the dealt ranges assume it, but a CTA this small would let the block
     // scheduler place two on one SM. Asking for more than half an SM's shared memory makes a second
     // resident CTA impossible.
@@ -585,7 +630,7 @@ __device__ __forceinline__ void stage_all(float4* src, const float4* bodies, int
 // Every lane of the CTA's used warps calls it (lanes of split s >= S contribute zero).
 __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLane& sl, bool active, int64_t tgt_first_src,
                                                int64_t tg, int64_t tcount, int L, int S, int S2, int64_t n, int chunk,
-                                               float eps2, float4* wpart) {
+                                               float eps2, float4* wpart, uint64_t* tbar, uint32_t parity) {
     Interact<2, true> it;
     it.zero_all();
     LIME_WTRACE(0);
@@ -594,8 +639,16 @@ __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLan
         for (int r = 0; r < 2; ++r) {
             int64_t t = tg + 2 * sl.p + r;
             t = t < tcount ? t : tcount - 1;
-            it.set(r, src[padded(static_cast<int>(tgt_first_src + t), L)]);
+            const int i = static_cast<int>(tgt_first_src + t);
+            if (tbar) mbar_wait(&tbar[(i / L) / kStageRows], parity);
+            it.set(r, src[padded(i, L)]);
         }
+        if (tbar) mbar_wait(&tbar[sl.s / kStageRows], parity);
+    }
+    // The lanes of a warp can leave the waits at different times; without this the warp runs the
+    // split loop once per lane subset (ncu r02, per-lane barriers: 1.44x the interactions issued).
+    __syncwarp();
+    if (active && sl.s < S) {
         const int64_t j0 = static_cast<int64_t>(sl.s) * L;
         split_sum(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
                   eps2);
@@ -635,17 +688,28 @@ struct SmallArgs {
     float4* accel;
     int S, S2, L, chunk;
     int64_t groups;
+    int tma;             // sources staged by TMA row boxes (map), else LDG
+    int rows;
 };
 
-__global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const __grid_constant__ SmallArgs a) {
+__global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const __grid_constant__ SmallArgs a,
+                                                                         const __grid_constant__ CUtensorMap map) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
-    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.S, a.L));   // [slots][blocks][4]
+    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.rows, a.L));   // [slots][blocks][4]
+    __shared__ __align__(8) uint64_t tbar[kMaxStageCopies];
     pdl_enter();
     const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
     const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
-    stage_all<false>(src, a.bodies, a.n_src, a.L);
-    __syncthreads();
+    if (a.tma) {
+        if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) mbar_init(&tbar[threadIdx.x], 1);
+        fence_mbar_init();
+        __syncthreads();
+        stage_tma(src, &map, a.S, a.L, tbar);
+    } else {
+        stage_all<false>(src, a.bodies, a.n_src, a.L);
+        __syncthreads();
+    }
     const SmallLane sl(a.S2);
     const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
     const int ct = static_cast<int>(threadIdx.x);
@@ -654,7 +718,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
     for (int64_t r0 = gb; r0 < ge; r0 += slots) {
         const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
         small_lane_sum(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
-                       a.S2, a.n_src, a.chunk, a.eps2, wpart);
+                       a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0);
         __syncthreads();
         const int64_t t = r0 * kGroupTargets + ct;
         if (ct < ng * kGroupTargets && t < a.tgt_count) a.accel[t] = small_target_sum(wpart, ct, a.S2);
@@ -678,8 +742,13 @@ static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream) {
     a.L = p.L;
     a.chunk = p.chunk;
     a.groups = p.groups;
+    a.tma = p.tma;
+    a.rows = p.rows;
+    CUtensorMap map;
+    std::memset(&map, 0, sizeof map);
+    if (a.tma && !make_rows_map(&map, f.bodies, p.S, p.L)) return cudaErrorInvalidValue;
     return launch_pdl(&force_small_kernel, dim3(static_cast<unsigned>(p.grid)), dim3(static_cast<unsigned>(p.block)),
-                      p.smem, stream, a);
+                      p.smem, stream, a, map);
 }
 
 // =====================================================================================
@@ -705,6 +774,7 @@ struct SimArgs {
     int32_t S, S2, L, chunk;
     int64_t groups;
     float eps2, dt;
+    int tma, rows;
 };
 
 __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target) {
@@ -721,10 +791,18 @@ __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target
 }
 
 
-__global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(const __grid_constant__ SimArgs a) {
+__global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(const __grid_constant__ SimArgs a,
+                                                                            const __grid_constant__ CUtensorMap map_pos,
+                                                                            const __grid_constant__ CUtensorMap map_alt) {
     extern __shared__ __align__(128) uint8_t small_smem[];
     float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
-    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.S, a.L));   // [slots][blocks][4]
+    float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.rows, a.L));   // [slots][blocks][4]
+    __shared__ __align__(8) uint64_t tbar[kMaxStageCopies];
+    if (a.tma) {
+        if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) mbar_init(&tbar[threadIdx.x], 1);
+        fence_mbar_init();
+        __syncthreads();
+    }
     const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
     const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
     const SmallLane sl(a.S2);
@@ -741,8 +819,15 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
         __syncthreads();
 #endif
         LIME_TRACE_AT(k, 5);
-        stage_all<true>(src, cur, a.n, a.L);       // what every CTA wrote in the previous step (L2)
-        __syncthreads();
+        if (a.tma) {
+            // the copies read what every CTA wrote in the previous step (generic-proxy stores,
+            // ordered before this point by the grid barrier's release/acquire): proxy fence first
+            if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) fence_proxy_async_global();
+            stage_tma(src, (k & 1) ? &map_alt : &map_pos, a.S, a.L, tbar);
+        } else {
+            stage_all<true>(src, cur, a.n, a.L);   // what every CTA wrote in the previous step (L2)
+            __syncthreads();
+        }
         LIME_TRACE_AT(k, 6);
         for (int64_t r0 = gb; r0 < ge; r0 += slots) {
             const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
@@ -751,12 +836,13 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
             if (owner) v = a.vel[t];                   // issued before the force work: latency hidden
             small_lane_sum(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
-                           a.eps2, wpart);
+                           a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1));
             LIME_TRACE_AT(k, 4);
             __syncthreads();
             LIME_TRACE_AT(k, 1);
             if (owner) {
                 const float4 acc = small_target_sum(wpart, ct, a.S2);
+                if (a.tma) mbar_wait(&tbar[(static_cast<int>(t) / a.L) / kStageRows], static_cast<uint32_t>(k & 1));
                 float4 pn = src[padded(static_cast<int>(t), a.L)];
                 v.x = fmaf(acc.x, a.dt, v.x);
                 v.y = fmaf(acc.y, a.dt, v.y);
@@ -841,6 +927,13 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.groups = p.groups;
     a.eps2 = eps2;
     a.dt = dt;
+    a.tma = p.tma;
+    a.rows = p.rows;
+    CUtensorMap map_pos, map_alt;
+    std::memset(&map_pos, 0, sizeof map_pos);
+    std::memset(&map_alt, 0, sizeof map_alt);
+    if (a.tma && (!make_rows_map(&map_pos, pos, p.S, p.L) || !make_rows_map(&map_alt, alt, p.S, p.L)))
+        return cudaErrorInvalidValue;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(static_cast<unsigned>(p.grid));
     cfg.blockDim = dim3(static_cast<unsigned>(p.block));
@@ -851,7 +944,7 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     at[0].val.cooperative = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, simulate_small_kernel, a);
+    e = cudaLaunchKernelEx(&cfg, simulate_small_kernel, a, map_pos, map_alt);
     if (e != cudaSuccess) return e;
     return cudaGetLastError();
 }

@@ -19,3 +19,7 @@ for k in $KERNELS; do
       -o gpurun_out/prof_${k}_${TAG} -f python tools/prof_kernels.py $k 2 > gpurun_out/prof_${k}_${TAG}.log 2>&1
   echo "prof $k rc=$?"
 done
+# summaries on the box (the .ncu-rep files of a full round exceed what gpurun brings back)
+mkdir -p gpurun_out/prof_${TAG}; PROF_DIR=gpurun_out/prof_${TAG} python tools/make_profiles.py ${TAG} > gpurun_out/prof_${TAG}/make_profiles.log 2>&1
+cp gpurun_out/launches_${TAG}.csv gpurun_out/bench_${TAG}.json gpurun_out/prof_${TAG}/ 2>/dev/null
+if [ -z "$KEEP_REPS" ]; then rm -f gpurun_out/prof_*_${TAG}.ncu-rep; fi
