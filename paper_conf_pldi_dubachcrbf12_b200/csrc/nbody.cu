@@ -575,8 +575,14 @@ static int small_smem_bound() {
 #ifdef LIME_TRACE
 __device__ long long g_lime_trace[kNumSMsB200 * 64 * 8];
 __device__ __forceinline__ unsigned smid() { unsigned r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
+__device__ __forceinline__ long long gtimer() { long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t; }
+#ifdef LIME_TRACE_GLOBAL
+#define LIME_CLOCK() gtimer()        // ns, comparable across SMs (tools/trace_barrier.py)
+#else
+#define LIME_CLOCK() clock64()
+#endif
 #define LIME_TRACE_AT(k, slot) \
-    do { if (threadIdx.x == 0 && (k) < 64) { g_lime_trace[(blockIdx.x * 64 + (k)) * 8 + (slot)] = clock64(); \
+    do { if (threadIdx.x == 0 && (k) < 64) { g_lime_trace[(blockIdx.x * 64 + (k)) * 8 + (slot)] = LIME_CLOCK(); \
          g_lime_trace[(blockIdx.x * 64 + (k)) * 8 + 7] = smid(); } } while (0)
 __device__ long long g_lime_wtrace[kNumSMsB200 * 32 * 2];   // step 20: per warp (data ready, lane sum done)
 __device__ int g_lime_step;
