@@ -878,6 +878,17 @@ def main():
     elif rank == 0:
         line["cpu_baseline"] = None
     line["peaks"] = peaks
+    # compact digest of every sub-line, LAST in the JSON line so that a driver keeping only the tail
+    # of stdout still sees each config's time and roofline fraction
+    digest = {}
+    for group in ("configs", "sharded_configs"):
+        for k, v in (line.get(group) or {}).items():
+            if isinstance(v, dict) and "roofline" in v:
+                t = v.get("ms_per_launch", v.get("ms_per_step", v.get("ms_per_call")))
+                digest[k] = {"ms": t if not isinstance(t, dict) else None, "value": v.get("value"),
+                             "unit": v.get("unit"), "frac": v["roofline"].get("frac"),
+                             "bound": v["roofline"].get("bound")}
+    line["digest"] = digest
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
