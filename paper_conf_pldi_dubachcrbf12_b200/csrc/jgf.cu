@@ -132,7 +132,15 @@ template <> __device__ __forceinline__ const double* series_sin<double>() { retu
 // inner term is ONE packed FFMA2 (re and im) and the only lane-divergent accesses are the R + 1024/R
 // table gathers per coefficient. R = 16 for both precisions (measured on B200: fp32 R = 16 at 62 regs,
 // 8 CTAs/SM: 24.7 us vs R = 32 at 96 regs: 28.9 us; fp64 R = 16 at 108 regs: 46.6 us).
-template <typename T, int R>
+// LIME_SERIES_SPLIT (A/B, tools/time_series.py r02): 1 = one coefficient per thread, whole warps per
+// grid-stride iteration (fp32 21.5 us, fp64 31.8 us; the previous per-thread loop: 25.5 / 40.0 us);
+// 2 / 4 threads per coefficient: 48 / 130 us fp32 -- lanes with different u ranges turn the node
+// weights' constant-bank loads lane-divergent, which serialises them.
+#ifndef LIME_SERIES_SPLIT
+#define LIME_SERIES_SPLIT 1
+#endif
+constexpr int kSeriesSplit = LIME_SERIES_SPLIT;
+template <typename T, int R, int SPLIT>
 __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_kernel(const __grid_constant__ SeriesNodes<T> G,
                                                               int64_t n0, int64_t count, T* __restrict__ out) {
     using T2 = typename Vec2<T>::type;
@@ -150,9 +158,16 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
     for (int i = threadIdx.x; i < kSeriesM; i += blockDim.x) { sc[series_pos(i)] = gc[i]; ss[series_pos(i)] = gs[i]; }
     __syncthreads();
     const T dx = static_cast<T>(2.0 / kSeriesM);
-    for (int64_t k = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; k < count;
-         k += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-        const int64_t n = n0 + k;
+    // SPLIT > 1: SPLIT consecutive lanes share coefficient k, each summing NU/SPLIT consecutive u
+    // blocks; partial sums added by a shuffle butterfly (whole warps iterate together)
+    const int h = static_cast<int>(threadIdx.x) % SPLIT;
+    constexpr int NUS = NU / SPLIT;
+    static_assert(NU % SPLIT == 0 && 32 % SPLIT == 0, "split must divide the u range and the warp");
+    for (int64_t base = blockIdx.x * static_cast<int64_t>(blockDim.x); base < count * SPLIT;
+         base += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t k = (base + threadIdx.x) / SPLIT;
+        const bool valid = k < count;
+        const int64_t n = n0 + (valid ? k : count - 1);
         const int step = static_cast<int>(n % kSeriesM);
         T2 V[R];                                      // V_v = e^{i theta (n v mod m)}
         int p = 0;
@@ -164,7 +179,7 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
             p -= (p >= kSeriesM) ? kSeriesM : 0;
         }
         const int step_u = p;                         // R n mod m
-        int q = 0;                                    // R n u mod m
+        int q = static_cast<int>((static_cast<int64_t>(step_u) * (h * NUS)) % kSeriesM);   // R n u mod m
         T a = 0, b = 0;
         // fp64: g_{Ru+v} for the next u is loaded one iteration ahead (the constant-bank loads at a
         // run-time offset otherwise stall the first DFMA of each chain; 46.4 -> 42.0 us). fp32 is
@@ -172,14 +187,14 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
         constexpr bool kAhead = sizeof(T) == 8;
         T gn[R];
 #pragma unroll
-        for (int v = 0; v < R; ++v) gn[v] = kAhead ? G.g[v] : T(0);
+        for (int v = 0; v < R; ++v) gn[v] = kAhead ? G.g[h * NUS * R + v] : T(0);
 #pragma unroll 1
-        for (int u = 0; u < NU; ++u) {
+        for (int u = h * NUS; u < (h + 1) * NUS; ++u) {
             T g[R];
 #pragma unroll
             for (int v = 0; v < R; ++v) g[v] = kAhead ? gn[v] : G.g[u * R + v];
             if constexpr (kAhead) {
-                const int un = u + 1 < NU ? u + 1 : u;
+                const int un = u + 1 < (h + 1) * NUS ? u + 1 : u;
 #pragma unroll
                 for (int v = 0; v < R; ++v) gn[v] = G.g[un * R + v];
             }
@@ -199,9 +214,16 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
             b = fma(ur, wi, b);
             b = fma(ui, wr, b);                       // Im(U W)
         }
-        if (n == 0) { a = a * static_cast<T>(0.5); b = 0; }   // a_0 = T[f] / 2, b_0 = 0
-        out[2 * k + 0] = a * dx;
-        out[2 * k + 1] = b * dx;
+#pragma unroll
+        for (int o = 1; o < SPLIT; o <<= 1) {
+            a += __shfl_xor_sync(0xffffffffu, a, o);
+            b += __shfl_xor_sync(0xffffffffu, b, o);
+        }
+        if (valid && h == 0) {
+            if (n == 0) { a = a * static_cast<T>(0.5); b = 0; }   // a_0 = T[f] / 2, b_0 = 0
+            out[2 * k + 0] = a * dx;
+            out[2 * k + 1] = b * dx;
+        }
     }
 }
 
@@ -213,8 +235,9 @@ static cudaError_t launch_series_t(int64_t n0, int64_t count, T* out, cudaStream
     cudaError_t e = series_tables_ready(stream);
     if (e != cudaSuccess) return e;
     int grid = launch_override().grid_ctas;
-    if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(count, kSeriesBlock), 16LL * device_num_sms()));
-    series_kernel<T, R><<<grid, kSeriesBlock, 0, stream>>>(series_nodes<T>(), n0, count, out);
+    if (grid <= 0)
+        grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(count * kSeriesSplit, kSeriesBlock), 16LL * device_num_sms()));
+    series_kernel<T, R, kSeriesSplit><<<grid, kSeriesBlock, 0, stream>>>(series_nodes<T>(), n0, count, out);
     return cudaGetLastError();
 }
 
