@@ -18,11 +18,15 @@ int nbody_variant() { return 0; }
 bool pdl_enabled() { return false; }
 cudaError_t ensure_dynamic_smem(const void*, int) { return cudaSuccess; }
 int cached_occupancy(const void*, int, size_t) { return 1; }
+void* tensor_map_encoder() { return nullptr; }
 }
 using namespace lime;
 using namespace lime::nbody;
 
-constexpr int kL = 128, kS = 32;
+#ifndef MB_L
+#define MB_L 128
+#endif
+constexpr int kL = MB_L, kS = 4096 / MB_L;
 
 template <int W, int Q, int LAYOUT>
 __global__ void __launch_bounds__(W * 32, 1) mb(const float4* __restrict__ bodies, int reps, long long* cyc, float4* out) {
@@ -32,7 +36,7 @@ __global__ void __launch_bounds__(W * 32, 1) mb(const float4* __restrict__ bodie
     int s;
     if (LAYOUT == 0) s = (warp + blockIdx.x) % kS;
     else if (LAYOUT == 1) s = (warp * 16 + lane / 2) % kS;
-    else s = lane;
+    else s = lane % kS;
     Interact<2 * Q, true> it;
 #pragma unroll
     for (int r = 0; r < 2 * Q; ++r) it.set(r, bodies[(blockIdx.x * 64 + threadIdx.x * 2 * Q + r) % 4096]);
@@ -48,8 +52,7 @@ __global__ void __launch_bounds__(W * 32, 1) mb(const float4* __restrict__ bodie
 }
 
 template <int W, int Q, int LAYOUT>
-void run(const float4* bodies, float4* out, long long* cyc) {
-    const int reps = 16;
+void run(const float4* bodies, float4* out, long long* cyc, int reps = 16) {
     const int smem = kS * (kL + 1) * 16;
     cudaFuncSetAttribute(mb<W, Q, LAYOUT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     mb<W, Q, LAYOUT><<<148, W * 32, smem>>>(bodies, reps, cyc, out);
@@ -63,9 +66,9 @@ void run(const float4* bodies, float4* out, long long* cyc) {
     const double lane_ops = double(W) * 32 * 2 * Q * kL * reps * 12;
     cudaFuncAttributes fa;
     cudaFuncGetAttributes(&fa, mb<W, Q, LAYOUT>);
-    printf("{\"W\": %d, \"Q\": %d, \"layout\": %d, \"regs\": %d, \"cycles_mean\": %.0f, \"fp32_pipe_eff\": %.3f, "
+    printf("{\"L\": %d, \"reps\": %d, \"W\": %d, \"Q\": %d, \"layout\": %d, \"regs\": %d, \"cycles_mean\": %.0f, \"fp32_pipe_eff\": %.3f, "
            "\"cycles_per_warp_source\": %.2f, \"err\": \"%s\"}\n",
-           W, Q, LAYOUT, fa.numRegs, mean, lane_ops / (128.0 * mean), mean / (double(reps) * kL * W / 4.0),
+           kL, reps, W, Q, LAYOUT, fa.numRegs, mean, lane_ops / (128.0 * mean), mean / (double(reps) * kL * W / 4.0),
            cudaGetErrorString(cudaGetLastError()));
 }
 
@@ -82,20 +85,11 @@ int main() {
     cudaMalloc(&out, 148 * 1024 * 4 * 16);
     cudaMalloc(&cyc, 148 * 8);
     cudaMemcpy(bodies, h.data(), 4096 * 16, cudaMemcpyHostToDevice);
-    run<14, 1, 1>(bodies, out, cyc);
-    run<14, 1, 0>(bodies, out, cyc);
-    run<16, 1, 0>(bodies, out, cyc);
-    run<16, 1, 1>(bodies, out, cyc);
-    run<28, 1, 1>(bodies, out, cyc);
-    run<32, 1, 0>(bodies, out, cyc);
-    run<7, 2, 2>(bodies, out, cyc);
-    run<7, 2, 0>(bodies, out, cyc);
-    run<8, 2, 0>(bodies, out, cyc);
-    run<14, 2, 0>(bodies, out, cyc);
-    run<14, 2, 1>(bodies, out, cyc);
-    run<16, 2, 0>(bodies, out, cyc);
-    run<4, 4, 0>(bodies, out, cyc);
-    run<7, 4, 0>(bodies, out, cyc);
-    run<8, 4, 0>(bodies, out, cyc);
+    for (int reps : {1, 2, 16}) {
+        run<28, 1, 1>(bodies, out, cyc, reps);
+        run<28, 1, 2>(bodies, out, cyc, reps);
+        run<14, 2, 1>(bodies, out, cyc, reps);
+        run<28, 2, 1>(bodies, out, cyc, reps);
+    }
     return 0;
 }
