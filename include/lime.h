@@ -153,6 +153,23 @@ lime_status lime_map_nbody_f64(const double *bodies, int64_t n_src, int64_t tgt_
 lime_status lime_map_nbody_integrate(float *pos, float *vel, const float *accel, int64_t n,
                                      float dt, void *stream);
 
+/* One N-Body step of a target shard with the integrator fused into the force map
+ * (the task graph's `computeForces => forceAccumulator` edge, PAPER.md L106-114;
+ * A9): for t in [0, tgt_count), with a_t the acceleration lime_map_nbody computes
+ * for target tgt_begin + t against all n_src bodies and p_t = bodies[tgt_begin + t],
+ *   vel[t].xyz += a_t.xyz * dt ;  pos_out[t] = p_t with .xyz += vel[t].xyz * dt
+ * (pos_out.w = p_t.w, vel.w kept) -- bit-identical to lime_map_nbody followed by
+ * lime_map_nbody_integrate on the shard, without materialising the accelerations
+ * (n_src <= 8192: one launch; larger: force map into ws, then the integrator).
+ * bodies [n_src][4], vel and pos_out [tgt_count][4] float, device, 16-B aligned,
+ * pairwise disjoint (pos_out is written out of place: the map reads every body).
+ * ws: lime_map_nbody_step_workspace_bytes(n_src, tgt_count) bytes, zeroed once.
+ * Errors as lime_map_nbody, plus LIME_ERR_ALIASING for overlapping vel/pos_out. */
+size_t lime_map_nbody_step_workspace_bytes(int64_t n_src, int64_t tgt_count);
+lime_status lime_map_nbody_step(const float *bodies, int64_t n_src, int64_t tgt_begin,
+                                int64_t tgt_count, float eps2, float dt, float *vel,
+                                float *pos_out, void *ws, size_t ws_bytes, void *stream);
+
 /* `steps` complete N-Body simulation steps on DEVICE buffers (the paper's task
  * graph run repeatedly, `particles => computeForces => forceAccumulator`,
  * PAPER.md L106-114; its 4096-body size, Table 3): per step the force map

@@ -7,7 +7,7 @@ workspaces. Every step of the path runs in the CUDA kernels; there is no CPU fal
 library is missing, load() raises.
 
 Public API (names follow the ABI):
-    map_nbody, map_nbody_integrate, nbody_simulate, nbody_simulate_host,
+    map_nbody, map_nbody_integrate, map_nbody_step, nbody_simulate, nbody_simulate_host,
     map_blackscholes, map_reduce_blackscholes_sum,
     map_mandelbrot, map_matmul_bf16,
     reduce_sum / reduce_min / reduce_max (f32, f64, i32, i64),
@@ -52,6 +52,8 @@ SIGNATURES = {
     "lime_nbody_splits": (_int, [_i64]),
     "lime_map_nbody": (_int, [_p, _i64, _i64, _i64, _f, _p, _p, _sz, _p]),
     "lime_map_nbody_integrate": (_int, [_p, _p, _p, _i64, _f, _p]),
+    "lime_map_nbody_step_workspace_bytes": (_sz, [_i64, _i64]),
+    "lime_map_nbody_step": (_int, [_p, _i64, _i64, _i64, _f, _f, _p, _p, _p, _sz, _p]),
     "lime_map_nbody_f64_workspace_bytes": (_sz, [_i64, _i64]),
     "lime_map_nbody_f64": (_int, [_p, _i64, _i64, _i64, C.c_double, _p, _p, _sz, _p]),
     "lime_nbody_simulate_workspace_bytes": (_sz, [_i64]),
@@ -235,6 +237,26 @@ def map_nbody_integrate(pos: torch.Tensor, vel: torch.Tensor, accel: torch.Tenso
     with torch.cuda.device(dev):
         _check(L.lime_map_nbody_integrate(pos.data_ptr(), vel.data_ptr(), accel.data_ptr(), n, dt, _stream(dev)),
                "lime_map_nbody_integrate")
+
+
+def map_nbody_step(bodies: torch.Tensor, eps2: float, dt: float, vel: torch.Tensor, tgt_begin: int = 0,
+                   tgt_count: int | None = None, out: torch.Tensor | None = None) -> torch.Tensor:
+    """Fused force map + integrator for targets [tgt_begin, tgt_begin+tgt_count): updates vel
+    ([count][4]) in place and returns the new positions ([count][4], out of place)."""
+    L = load()
+    _dev_tensor(bodies, torch.float32, "bodies", 4)
+    n = bodies.shape[0]
+    tgt_count = _target_range(n, tgt_begin, tgt_count)
+    dev = bodies.device
+    _dev_tensor(vel, torch.float32, "vel", 4, numel=4 * tgt_count, device=dev)
+    if out is None:
+        out = torch.empty((tgt_count, 4), dtype=torch.float32, device=dev)
+    _dev_tensor(out, torch.float32, "out", 4, numel=4 * tgt_count, device=dev)
+    with torch.cuda.device(dev):
+        ws = workspace(dev, "nbody_step", L.lime_map_nbody_step_workspace_bytes(n, tgt_count))
+        _check(L.lime_map_nbody_step(bodies.data_ptr(), n, tgt_begin, tgt_count, eps2, dt, vel.data_ptr(),
+                                     out.data_ptr(), ws.data_ptr(), ws.numel(), _stream(dev)), "lime_map_nbody_step")
+    return out
 
 
 def nbody_simulate(pos: torch.Tensor, vel: torch.Tensor, steps: int, eps2: float, dt: float) -> None:

@@ -248,6 +248,36 @@ lime_status lime_map_nbody_integrate(float* pos, float* vel, const float* accel,
                     "lime_map_nbody_integrate");
 }
 
+size_t lime_map_nbody_step_workspace_bytes(int64_t n_src, int64_t tgt_count) {
+    if (n_src < 0 || tgt_count < 0) return 0;
+    return nbody::step_workspace_bytes(n_src, tgt_count);
+}
+
+lime_status lime_map_nbody_step(const float* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count, float eps2,
+                                float dt, float* vel, float* pos_out, void* ws, size_t ws_bytes, void* stream) {
+    if (n_src < 0 || tgt_begin < 0 || tgt_count < 0 || tgt_begin > n_src || tgt_count > n_src - tgt_begin)
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_step: shard [%lld, %lld+%lld) outside [0, %lld)",
+                    (long long)tgt_begin, (long long)tgt_begin, (long long)tgt_count, (long long)n_src);
+    if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f) || !std::isfinite(dt))
+        return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_step: eps2 must be finite and >= FLT_MIN, dt finite");
+    if (tgt_count == 0) return LIME_OK;
+    if (!bodies || !vel || !pos_out || !ws) return fail(LIME_ERR_INVALID_ARG, "lime_map_nbody_step: null pointer");
+    if (!aligned16(bodies) || !aligned16(vel) || !aligned16(pos_out) || !aligned16(ws))
+        return fail(LIME_ERR_MISALIGNED, "lime_map_nbody_step: bodies, vel, pos_out and ws must be 16-byte aligned");
+    const size_t tb = static_cast<size_t>(tgt_count) * 16, nb = static_cast<size_t>(n_src) * 16;
+    if (overlap(pos_out, tb, bodies, nb) || overlap(vel, tb, bodies, nb) || overlap(vel, tb, pos_out, tb))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody_step: bodies, vel and pos_out must be disjoint");
+    if (overlap(ws, ws_bytes, bodies, nb) || overlap(ws, ws_bytes, vel, tb) || overlap(ws, ws_bytes, pos_out, tb))
+        return fail(LIME_ERR_ALIASING, "lime_map_nbody_step: workspace overlaps an operand");
+    LIME_TRY(check_device());
+    const size_t need = nbody::step_workspace_bytes(n_src, tgt_count);
+    if (ws_bytes < need) return fail(LIME_ERR_WORKSPACE, "lime_map_nbody_step: workspace %zu B < %zu B", ws_bytes, need);
+    return launched(nbody::launch_step(reinterpret_cast<const float4*>(bodies), n_src, tgt_begin, tgt_count, eps2, dt,
+                                       reinterpret_cast<float4*>(vel), reinterpret_cast<float4*>(pos_out), ws,
+                                       static_cast<cudaStream_t>(stream)),
+                    "lime_map_nbody_step");
+}
+
 static lime_status sim_validate(const char* fn, int64_t n, int32_t steps, float eps2, float dt) {
     if (n < 0 || steps < 0) return fail(LIME_ERR_INVALID_ARG, "%s: n or steps < 0", fn);
     if (!(std::isfinite(eps2) && eps2 >= 1.17549435e-38f) || !std::isfinite(dt))

@@ -45,6 +45,9 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
                          float eps2, float4* accel, void* ws, cudaStream_t stream);
 cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int64_t n, float dt,
                              cudaStream_t stream);
+size_t step_workspace_bytes(int64_t n_src, int64_t tgt_count);
+cudaError_t launch_step(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count, float eps2,
+                        float dt, float4* vel, float4* pos_out, void* ws, cudaStream_t stream);
 size_t simulate_workspace_bytes(int64_t n);
 cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, float eps2, float dt, void* ws,
                             cudaStream_t stream);

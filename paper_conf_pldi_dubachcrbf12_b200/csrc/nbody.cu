@@ -696,6 +696,10 @@ struct SmallArgs {
     int64_t groups;
     int tma;             // sources staged by TMA row boxes (map), else LDG
     int rows;
+    // fused step (lime_map_nbody_step): integrate the targets instead of storing accel
+    float4* vel;         // [tgt_count] in/out, or null (force map only)
+    float4* pos_out;     // [tgt_count]
+    float dt;
 };
 
 __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const __grid_constant__ SmallArgs a,
@@ -727,12 +731,31 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
                        a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0);
         __syncthreads();
         const int64_t t = r0 * kGroupTargets + ct;
-        if (ct < ng * kGroupTargets && t < a.tgt_count) a.accel[t] = small_target_sum(wpart, ct, a.S2);
+        if (ct < ng * kGroupTargets && t < a.tgt_count) {
+            const float4 acc = small_target_sum(wpart, ct, a.S2);
+            if (a.vel == nullptr) {
+                a.accel[t] = acc;
+            } else {                                   // integrate_kernel's arithmetic on the old position
+                const int i = static_cast<int>(a.tgt_begin + t);
+                if (a.tma) mbar_wait(&tbar[(i / a.L) / kStageRows], 0);
+                float4 p = src[padded(i, a.L)];
+                float4 v = a.vel[t];
+                v.x = fmaf(acc.x, a.dt, v.x);
+                v.y = fmaf(acc.y, a.dt, v.y);
+                v.z = fmaf(acc.z, a.dt, v.z);
+                p.x = fmaf(v.x, a.dt, p.x);
+                p.y = fmaf(v.y, a.dt, p.y);
+                p.z = fmaf(v.z, a.dt, p.z);
+                a.vel[t] = v;
+                a.pos_out[t] = p;
+            }
+        }
         __syncthreads();                               // wpart[] is reused by the next round
     }
 }
 
-static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream) {
+static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream, float4* vel = nullptr, float4* pos_out = nullptr,
+                                float dt = 0.f) {
     const SmallPlan p = small_plan(f.n_src, f.tgt_count, device_num_sms());
     cudaError_t e = ensure_dynamic_smem(reinterpret_cast<const void*>(&force_small_kernel), small_smem_bound());
     if (e != cudaSuccess) return e;
@@ -750,6 +773,9 @@ static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream) {
     a.groups = p.groups;
     a.tma = p.tma;
     a.rows = p.rows;
+    a.vel = vel;
+    a.pos_out = pos_out;
+    a.dt = dt;
     CUtensorMap map;
     std::memset(&map, 0, sizeof map);
     if (a.tma && !make_rows_map(&map, f.bodies, p.S, p.L)) return cudaErrorInvalidValue;
@@ -1188,6 +1214,59 @@ __global__ void __launch_bounds__(256) integrate_kernel(float4* __restrict__ pos
         vel[i] = v;
         pos[i] = p;
     }
+}
+
+// Fused step tail for n_src > kSmallMaxSources (lime_map_nbody_step): the integrator on targets
+// [tgt_begin, tgt_begin + count), reading the old positions from `bodies` and writing pos_out.
+__global__ void __launch_bounds__(256) integrate_out_kernel(const float4* __restrict__ bodies, int64_t tgt_begin,
+                                                            float4* __restrict__ vel, const float4* __restrict__ accel,
+                                                            float4* __restrict__ pos_out, int64_t n, float dt) {
+    pdl_enter();
+    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const float4 a = ld_stream_f4(accel + i);
+        float4 v = vel[i];
+        float4 p = __ldg(bodies + tgt_begin + i);
+        v.x = fmaf(a.x, dt, v.x);
+        v.y = fmaf(a.y, dt, v.y);
+        v.z = fmaf(a.z, dt, v.z);
+        p.x = fmaf(v.x, dt, p.x);
+        p.y = fmaf(v.y, dt, p.y);
+        p.z = fmaf(v.z, dt, p.z);
+        vel[i] = v;
+        pos_out[i] = p;
+    }
+}
+
+// workspace: [force workspace][accel, tgt_count x 16 B] (the accel part only for n_src > 8192)
+static size_t step_accel_offset(int64_t n_src, int64_t tgt_count) {
+    return ((workspace_bytes(n_src, tgt_count) + 255) / 256) * 256;
+}
+size_t step_workspace_bytes(int64_t n_src, int64_t tgt_count) {
+    return step_accel_offset(n_src, tgt_count) + (n_src > kSmallMaxSources ? static_cast<size_t>(tgt_count) * 16 : 0);
+}
+
+cudaError_t launch_step(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count, float eps2,
+                        float dt, float4* vel, float4* pos_out, void* ws, cudaStream_t stream) {
+    if (tgt_count == 0) return cudaSuccess;
+    const LaunchOverride& ov = launch_override();
+    if (nbody_variant() == 0 && n_src <= kSmallMaxSources && ov.block_threads == 0 && ov.per_thread == 0) {
+        ForceArgs a;                                   // the small-N kernel with the integrator fused in
+        a.bodies = bodies;
+        a.n_src = n_src;
+        a.tgt_begin = tgt_begin;
+        a.tgt_count = tgt_count;
+        a.eps2 = eps2;
+        a.accel = nullptr;
+        return launch_small(a, stream, vel, pos_out, dt);
+    }
+    float4* accel = reinterpret_cast<float4*>(static_cast<char*>(ws) + step_accel_offset(n_src, tgt_count));
+    cudaError_t e = launch_force(bodies, n_src, tgt_begin, tgt_count, eps2, accel, ws, stream);
+    if (e != cudaSuccess) return e;
+    int grid = ov.grid_ctas;
+    if (grid <= 0) grid = static_cast<int>(mn<int64_t>(ceil_div<int64_t>(tgt_count, 256), 8LL * device_num_sms()));
+    return launch_pdl(&integrate_out_kernel, dim3(grid), dim3(256), 0, stream, bodies, tgt_begin, vel,
+                      static_cast<const float4*>(accel), pos_out, tgt_count, dt);
 }
 
 cudaError_t launch_integrate(float4* pos, float4* vel, const float4* accel, int64_t n, float dt,

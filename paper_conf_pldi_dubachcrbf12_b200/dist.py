@@ -75,11 +75,17 @@ class NBodySim:
         # after the map has run), so there is no exchange and no copy
         self.pos_full = self.pos if self.world == 1 else torch.empty((n, 4), dtype=torch.float32, device=self.device)
         self.accel = torch.empty_like(self.pos)
+        # the CUDA path fuses the integrator into the force map (lime_map_nbody_step): one launch per
+        # step at n <= 8192, no accelerations in memory. It writes the new shard positions out of
+        # place: into pos_alt (then swapped) at one rank, where the map reads the shard itself.
+        self.fused = force_fn is None and integrate_fn is None
         if force_fn is None or integrate_fn is None:
             import paper_conf_pldi_dubachcrbf12_b200 as lime
             force_fn = force_fn or (lambda p, b, c, e, out: lime.map_nbody(p, e, b, c, out=out))
             integrate_fn = integrate_fn or lime.map_nbody_integrate
+            self._step_fn = lime.map_nbody_step
         self.force_fn, self.integrate_fn = force_fn, integrate_fn
+        self.pos_alt = torch.empty_like(self.pos) if (self.fused and self.world == 1) else None
 
     def gather(self):
         if self.world > 1:
@@ -88,6 +94,14 @@ class NBodySim:
     def step(self):
         """One task-graph pass: exchange, force map, integrate."""
         self.gather()
+        if self.fused:
+            if self.world == 1:
+                self._step_fn(self.pos, self.eps2, self.dt, self.vel, 0, self.count, out=self.pos_alt)
+                self.pos, self.pos_alt = self.pos_alt, self.pos
+                self.pos_full = self.pos
+            else:
+                self._step_fn(self.pos_full, self.eps2, self.dt, self.vel, self.begin, self.count, out=self.pos)
+            return
         self.force_fn(self.pos_full, self.begin, self.count, self.eps2, self.accel)
         self.integrate_fn(self.pos, self.vel, self.accel, self.dt)
 
@@ -105,6 +119,8 @@ class NBodySim:
         without launch gaps -- the paper's repeated task-graph passes (L113-114) as one launch."""
         if self.world != 1:
             raise RuntimeError("graph capture of the multi-rank step (NCCL inside the graph) is not supported")
+        if self.fused and steps % 2:
+            raise ValueError("capture an even number of steps (the fused step ping-pongs two position buffers)")
         s = torch.cuda.Stream(self.device)
         s.wait_stream(torch.cuda.current_stream(self.device))
         with torch.cuda.stream(s):

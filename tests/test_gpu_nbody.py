@@ -165,7 +165,7 @@ def test_nbody_f64_shards_and_config5_sample(lime):
 
 def test_cuda_graph_replay_matches_eager_steps(lime):
     from paper_conf_pldi_dubachcrbf12_b200 import dist as ldist
-    n, steps = 4096, 5
+    n, steps = 4096, 6                              # even: the fused step ping-pongs two buffers
     bodies = torch.from_numpy(inputs.nbody_bodies(n, seed=61))
     eager = ldist.NBodySim(bodies, 1e-4, 1e-3, "cuda:0")
     for _ in range(steps + 1):                      # capture() runs one warm-up step first
@@ -321,3 +321,42 @@ def test_mass_uniform_edge_masses(lime):
     ref0, mag0 = oracle.nbody_accel_rows(b, EPS2, rows, threads=8)
     assert np.all(np.isfinite(acc0))
     assert nbody_rel_err(acc0[rows], ref0, mag0).max() <= NBODY_RTOL
+
+
+@pytest.mark.parametrize("n", [31, 1000, 4096, 4097, 8192, 8193, 20000])
+def test_fused_step_matches_map_then_integrate(lime, n):
+    # lime_map_nbody_step (force map with the integrator fused in, out-of-place positions) is
+    # bit-identical to lime_map_nbody + lime_map_nbody_integrate, whole range and shards
+    b = inputs.nbody_bodies(n, seed=90 + n)
+    v0 = (inputs.nbody_bodies(n, seed=91 + n) * np.float32(0.05)).astype(np.float32)
+    v0[:, 3] = 0
+    for begin, count in [(0, n), (n // 3, n // 2), (n - 1, 1)]:
+        pos, vel = _dev(b), _dev(v0)
+        acc = lime.map_nbody(pos, float(EPS2), begin, count)
+        p_ref = pos[begin:begin + count].clone()
+        v_ref = vel[begin:begin + count].clone()
+        lime.map_nbody_integrate(p_ref, v_ref, acc, 1e-3)
+        v = vel[begin:begin + count].clone()
+        p_new = lime.map_nbody_step(pos, float(EPS2), 1e-3, v, begin, count)
+        assert torch.equal(p_new, p_ref) and torch.equal(v, v_ref), (n, begin, count)
+        assert torch.equal(pos, _dev(b))                              # sources untouched
+
+
+def test_fused_step_rejects_aliasing(lime):
+    pos = _dev(inputs.nbody_bodies(256, seed=3))
+    vel = torch.zeros_like(pos)
+    with pytest.raises(lime.LimeError):
+        lime.map_nbody_step(pos, float(EPS2), 1e-3, vel, out=pos)        # out of place only
+
+
+def test_graph_of_fused_steps_matches_eager(lime):
+    from paper_conf_pldi_dubachcrbf12_b200 import dist as ldist
+    n = 4096
+    b = torch.from_numpy(inputs.nbody_bodies(n, seed=95))
+    sim = ldist.NBodySim(b, float(EPS2), 1e-3, "cuda")
+    g = sim.capture(10)                                               # includes one warm-up step
+    g.replay()
+    torch.cuda.synchronize()
+    pos, vel = _dev(b.numpy()), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
+    _eager_steps(lime, pos, vel, 11)
+    assert torch.equal(sim.pos, pos) and torch.equal(sim.vel, vel)
