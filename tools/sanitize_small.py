@@ -27,6 +27,17 @@ def main():
     lime.nbody_simulate(p, v, 3, 1e-4, 1e-3)                  # persistent cooperative kernel
     lime.map_nbody_integrate(p, v, lime.map_nbody(p, 1e-4), 1e-3)
     lime.map_nbody_f64(b.double(), 1e-4)
+    # round 2: TMA row-box staging (n % 64 == 0), the fused step (small and general n), the
+    # 8192-body LDG staging and the persistent kernel on the TMA path
+    t = torch.from_numpy(inputs.nbody_bodies(1024, seed=4)).to(dev)
+    lime.map_nbody(t, 1e-4, 100, 333)
+    vt = torch.zeros((333, 4), dtype=torch.float32, device=dev)
+    lime.map_nbody_step(t, 1e-4, 1e-3, vt, 100, 333)
+    lime.map_nbody_step(big, 1e-4, 1e-3, torch.zeros((700, 4), dtype=torch.float32, device=dev), 0, 700)
+    e8 = torch.from_numpy(inputs.nbody_bodies(8192, seed=5)).to(dev)
+    lime.map_nbody(e8, 1e-4, 0, 257)
+    pt, vv = t.clone(), torch.zeros_like(t)
+    lime.nbody_simulate(pt, vv, 3, 1e-4, 1e-3)
     S, X, T = (torch.from_numpy(a).to(dev) for a in inputs.blackscholes_options(4099, seed=3))
     lime.map_blackscholes(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
     lime.map_reduce_blackscholes_sum(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
@@ -34,6 +45,8 @@ def main():
     A = torch.from_numpy(inputs.bf16_uniform(300, 136, 4, 0).view(np.int16)).to(dev).view(torch.bfloat16)
     B = torch.from_numpy(inputs.bf16_uniform(260, 136, 4, 1).view(np.int16)).to(dev).view(torch.bfloat16)
     lime.map_matmul_bf16(A, B)
+    B2 = torch.from_numpy(inputs.bf16_uniform(1030, 136, 4, 2).view(np.int16)).to(dev).view(torch.bfloat16)
+    lime.map_matmul_bf16(A, B2)                               # 256 x 512 pair tile, ragged M and N
     x = torch.randn(100003, device=dev)
     lime.reduce_sum(x), lime.reduce_min(x), lime.reduce_max(x)
     atoms = torch.from_numpy(inputs.cp_atoms(300)).to(dev)
