@@ -16,6 +16,10 @@
 #include "common.cuh"
 #include "kernels.h"
 
+#ifndef LIME_MANDEL_LAZY
+#define LIME_MANDEL_LAZY 16       // lazy-test block length (0: test every iteration)
+#endif
+
 namespace lime {
 namespace mandel {
 
@@ -69,7 +73,82 @@ struct State {
     }
 };
 
-template <int LW, int UNROLL>
+// Lazy escape test (round 2). R7 tests x^2 + y^2 <= 4 before every update; the test costs one
+// packed op of the 7 and the count/predicate bookkeeping. Escape is permanent: once |z_j|^2 > 4 with
+// |c| <= 1.9, |z_{j+1}| >= |z_j|^2 - |c| - (rounding, < 1e-5) > 2.09, and |z| grows from then on
+// (overflow gives inf/NaN, which fails the test too). So for such c the update can run B
+// iterations without tests, carrying x^2 and y^2 (6 packed ops per iteration, the same IEEE ops as
+// R7), and one test at the block end decides: pass -> all B tests of the block passed (count += B);
+// fail -> the pixel escaped inside the block: it stops counting, keeps the block-start state, and
+// after the warp's loop replays at most B TESTED iterations from that state to find the exact
+// escape iteration. Bit-identical to the tested loop; warps with any |c|^2 > 3.6 (the margin covers
+// the fp32 evaluation of |c|^2) take the tested loop.
+struct Lazy {
+    float2 x, y, xx, yy, cx, cy;
+    __device__ __forceinline__ void fast() {         // R7's update, no test; xx, yy = squares of (x, y)
+        const float2 z = bcast2(-0.0f), one = bcast2(1.0f), mone = bcast2(-1.0f);
+        const float2 xy = fma2(x, y, z);
+        x = fma2(fma2(yy, mone, xx), one, cx);
+        y = fma2(xy, bcast2(2.0f), cy);
+        xx = fma2(x, x, z);
+        yy = fma2(y, y, z);
+    }
+};
+
+// The tested loop from `st` until the warp has no live pixel or max_iter: returns via st.
+template <int UNROLL>
+__device__ __forceinline__ void tested_loop(State& st, int32_t it, int32_t max_iter) {
+    while (it + UNROLL <= max_iter) {
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) st.step();
+        it += UNROLL;
+        if (!__any_sync(0xffffffffu, st.a0 || st.a1)) return;
+    }
+    if (__any_sync(0xffffffffu, st.a0 || st.a1)) {
+        for (; it < max_iter; ++it) st.step();
+    }
+}
+
+template <int B>
+__device__ __forceinline__ void lazy_loop(State& st, int32_t max_iter) {
+    Lazy L;
+    L.x = st.x; L.y = st.y; L.cx = st.cx; L.cy = st.cy;
+    const float2 z = bcast2(-0.0f), one = bcast2(1.0f);
+    L.xx = fma2(L.x, L.x, z);
+    L.yy = fma2(L.y, L.y, z);
+    float2 xs = L.x, ys = L.y;                        // block-start state of a pixel that escaped
+    bool e0 = false, e1 = false;                      // escaped inside a lazy block, count pending
+    int32_t it = 0;
+    while (it + B <= max_iter) {
+        if (st.a0) { xs.x = L.x.x; ys.x = L.y.x; }
+        if (st.a1) { xs.y = L.x.y; ys.y = L.y.y; }
+#pragma unroll
+        for (int u = 0; u < B; ++u) L.fast();
+        const float2 s = fma2(L.xx, one, L.yy);       // the test of iteration it + B
+        if (st.a0) { if (s.x <= 4.0f) st.n0 += B; else { st.a0 = false; e0 = true; } }
+        if (st.a1) { if (s.y <= 4.0f) st.n1 += B; else { st.a1 = false; e1 = true; } }
+        it += B;
+        if (!__any_sync(0xffffffffu, st.a0 || st.a1)) break;
+    }
+    // pixels still live at it + B > max_iter: finish with tested iterations from where they are
+    if (__any_sync(0xffffffffu, st.a0 || st.a1)) {
+        st.x = L.x; st.y = L.y;
+        for (; it < max_iter; ++it) st.step();
+    }
+    // escaped pixels: replay their escape block with tests (<= B iterations, stops at the escape)
+    if (__any_sync(0xffffffffu, e0 || e1)) {
+        State r = st;
+        r.x = xs; r.y = ys;
+        r.n0 = 0; r.n1 = 0;
+        r.a0 = e0; r.a1 = e1;
+#pragma unroll 4
+        for (int u = 0; u < B; ++u) r.step();
+        if (e0) st.n0 += r.n0;
+        if (e1) st.n1 += r.n1;
+    }
+}
+
+template <int LW, int UNROLL, int LAZY>
 __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Args a) {
     constexpr int kTileW = 2 * LW, kTileH = 32 / LW;
     const unsigned lane = lane_id();
@@ -95,16 +174,15 @@ __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Arg
         st.n0 = st.n1 = 0;
         st.a0 = st.a1 = true;
 
-        int32_t it = 0;
-        while (it + UNROLL <= a.max_iter) {
-#pragma unroll
-            for (int u = 0; u < UNROLL; ++u) st.step();
-            it += UNROLL;
-            if (!__any_sync(0xffffffffu, st.a0 || st.a1)) break;
+        bool lazy = false;
+        if constexpr (LAZY > 0) {                     // every |c| of the warp <= 1.9 (|c|^2 <= 3.6)
+            // (uncontracted scalar ops: the SASS guard admits only R7's exact FFMA forms)
+            const float c2x = add_rn(mul_rn(st.cx.x, st.cx.x), mul_rn(st.cy.x, st.cy.x));
+            const float c2y = add_rn(mul_rn(st.cx.y, st.cx.y), mul_rn(st.cy.y, st.cy.y));
+            lazy = __all_sync(0xffffffffu, c2x <= 3.6f && c2y <= 3.6f);
         }
-        if (__any_sync(0xffffffffu, st.a0 || st.a1)) {
-            for (; it < a.max_iter; ++it) st.step();
-        }
+        if (lazy) lazy_loop<(LAZY > 0 ? LAZY : 1)>(st, a.max_iter);
+        else tested_loop<UNROLL>(st, 0, a.max_iter);
         int32_t* row = a.counts + static_cast<int64_t>(k) * a.width;
         if (v0) row[col] = st.n0;
         if (v1) row[col + 1] = st.n1;
@@ -119,19 +197,19 @@ __global__ void __launch_bounds__(256) mandel_kernel(const __grid_constant__ Arg
     }
 }
 
-template <int LW, int UNROLL>
+template <int LW, int UNROLL, int LAZY = 0>
 static cudaError_t launch_t(Args& a, cudaStream_t stream) {
     a.tiles_x = ceil_div<int32_t>(a.width, 2 * LW);
     a.ntiles = static_cast<int64_t>(a.tiles_x) * ceil_div<int32_t>(a.row_count, 32 / LW);
     int grid = launch_override().grid_ctas;
     if (grid <= 0) {
-        const int per_sm = mx(1, cached_occupancy(reinterpret_cast<const void*>(&mandel_kernel<LW, UNROLL>), 256, 0));
+        const int per_sm = mx(1, cached_occupancy(reinterpret_cast<const void*>(&mandel_kernel<LW, UNROLL, LAZY>), 256, 0));
         grid = per_sm * device_num_sms();
         const int64_t need = ceil_div<int64_t>(a.ntiles, 8);
         if (need < grid) grid = static_cast<int>(need);
     }
     a.total_warps = static_cast<unsigned>(grid) * 8u;
-    mandel_kernel<LW, UNROLL><<<grid, 256, 0, stream>>>(a);
+    mandel_kernel<LW, UNROLL, LAZY><<<grid, 256, 0, stream>>>(a);
     return cudaGetLastError();
 }
 
@@ -162,7 +240,10 @@ cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t
         case 7: return launch_t<4, 32>(a, stream);
         case 8: return launch_t<8, 64>(a, stream);
         case 1: return launch_t<8, 16>(a, stream);
-        default: return launch_t<4, 32>(a, stream);   // = case 7 (tools/tune_mandel.py: 3.19 vs 3.22 ms for 16x4/16)
+        case 9: return launch_t<4, 32, 16>(a, stream);
+        case 10: return launch_t<4, 32, 32>(a, stream);
+        case 11: return launch_t<4, 32, 8>(a, stream);
+        default: return launch_t<4, 32, LIME_MANDEL_LAZY>(a, stream);   // 8x8 tiles, vote every 32 (tools/tune_mandel.py)
     }
 }
 

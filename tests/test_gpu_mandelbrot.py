@@ -50,3 +50,23 @@ def test_full_frame_config3(lime):
     assert int(gpu.sum(dtype=np.int64)) == f["checksum"]
     again = lime.map_mandelbrot(W, H, f["x0"], f["y0"], f["dx"], f["dy"], f["max_iter"]).cpu().numpy()
     assert np.array_equal(gpu, again)
+
+
+@pytest.mark.parametrize("x0,y0,w,h,span,max_iter", [
+    (-1.95, -0.05, 200, 100, 0.1, 3000),      # |c| straddles 1.9: lazy and tested warps side by side
+    (0.2, -0.05, 256, 128, 0.1, 5000),        # near the cusp c = 1/4: long, slowly escaping orbits
+    (-0.75, 0.05, 256, 64, 0.02, 4000),       # the neck between the cardioid and the period-2 bulb
+    (-2.0, -1.5, 97, 61, 3.0, 1000),          # whole region, ragged tiles, max_iter not a block multiple
+])
+def test_lazy_escape_test_bit_exact(lime, x0, y0, w, h, span, max_iter):
+    # round 2: warps whose |c| <= 1.9 skip the per-iteration test and replay the escape block
+    # (DESIGN.md §5.4); the default kernel must equal the always-tested loop (launch override
+    # per_thread=7) and the oracle bit for bit
+    dx, dy = span / w, span / w
+    gpu = lime.map_mandelbrot(w, h, x0, y0, dx, dy, max_iter).cpu().numpy()
+    with lime.launch_override(per_thread=7):
+        tested = lime.map_mandelbrot(w, h, x0, y0, dx, dy, max_iter).cpu().numpy()
+    ref = oracle.mandelbrot(w, h, 0, 1, h, float(np.float32(x0)), float(np.float32(y0)), float(np.float32(dx)),
+                            float(np.float32(dy)), max_iter, threads=os.cpu_count() or 1)
+    assert np.array_equal(gpu, tested)
+    assert np.array_equal(gpu, ref)
