@@ -72,6 +72,21 @@ def test_nbody_validation_order(L):
     assert b"overlaps" in L.lime_last_error()
 
 
+def test_nbody_step_validation(L):
+    # lime_map_nbody_step (round 2): arguments -> alignment -> aliasing -> device, like lime_map_nbody
+    f = L.lime_map_nbody_step
+    wsb = L.lime_map_nbody_step_workspace_bytes(10, 10)
+    assert wsb >= L.lime_map_nbody_workspace_bytes(10, 10)
+    assert L.lime_map_nbody_step_workspace_bytes(1 << 20, 1 << 17) >= (1 << 17) * 16   # accel for the general path
+    assert f(A0, 10, 5, 6, 1e-4, 1e-3, A1, A1 + 512, WS, wsb, None) == 1          # shard outside [0, n)
+    assert f(A0, 10, 0, 10, 1e-4, float("nan"), A1, A1 + 512, WS, wsb, None) == 1  # dt not finite
+    assert f(A0, 10, 0, 0, 1e-4, 1e-3, A1, A1 + 512, WS, wsb, None) == 0          # empty shard: no-op
+    assert f(A0, 10, 0, 10, 1e-4, 1e-3, None, A1 + 512, WS, wsb, None) == 1       # null vel
+    assert f(A0, 10, 0, 10, 1e-4, 1e-3, A1 + 8, A1 + 512, WS, wsb, None) == 2     # misaligned vel
+    assert f(A0, 10, 0, 10, 1e-4, 1e-3, A1, A0 + 16, WS, wsb, None) == 3          # pos_out overlaps bodies
+    assert f(A0, 10, 0, 10, 1e-4, 1e-3, A1, A1 + 64, WS, wsb, None) == 3          # vel overlaps pos_out
+
+
 def test_integrate_and_bs_validation(L):
     assert L.lime_map_nbody_integrate(A0, A0 + 64, A1, 8, 1e-3, None) == 3      # pos/vel overlap
     assert L.lime_map_nbody_integrate(A0, A1, WS, 8, float("inf"), None) == 1   # dt not finite
