@@ -360,3 +360,22 @@ def test_graph_of_fused_steps_matches_eager(lime):
     pos, vel = _dev(b.numpy()), torch.zeros((n, 4), dtype=torch.float32, device="cuda")
     _eager_steps(lime, pos, vel, 11)
     assert torch.equal(sim.pos, pos) and torch.equal(sim.vel, vel)
+
+
+@pytest.mark.parametrize("n", [64, 128, 1088, 2112, 4032])
+def test_tma_staged_sizes_match_general_kernel(lime, n):
+    # n % 64 == 0 (n <= 4096) stages the sources with TMA row boxes of 16 splits; S = n / 64 not a
+    # multiple of 16 leaves zero-filled rows in the last box. Forces must equal the general
+    # kernel (launch override) bit for bit, on shards too, and the persistent simulation the
+    # eager fused steps.
+    b = _dev(inputs.nbody_bodies(n, seed=200 + n))
+    full = lime.map_nbody(b, float(EPS2))
+    with lime.launch_override(block_threads=128, per_thread=2):
+        assert torch.equal(lime.map_nbody(b, float(EPS2)), full)
+    begin, count = n // 5, n // 2
+    assert torch.equal(lime.map_nbody(b, float(EPS2), begin, count), full[begin:begin + count])
+    pos, vel = b.clone(), torch.zeros_like(b)
+    lime.nbody_simulate(pos, vel, 3, float(EPS2), 1e-3)
+    pe, ve = b.clone(), torch.zeros_like(b)
+    _eager_steps(lime, pe, ve, 3)
+    assert torch.equal(pos, pe) and torch.equal(vel, ve)

@@ -8,6 +8,7 @@
 //   variant 4: no __threadfence (red.release only); 5: + relaxed polling and one acquire fence;
 //   6: fence.acq_rel instead of __threadfence; 7: as 5 with ld.volatile polling
 //   8/9/10: two-level counter, 16/8/32 groups
+//   11/12: counter + broadcast go-flags (each CTA polls its own line; acquire / relaxed+fence)
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o tools/barrier_mb tools/barrier_mb.cu
 #include <cstdio>
 #include <cstdint>
@@ -17,6 +18,32 @@
 template <int V>
 __device__ __forceinline__ void gbar(unsigned* cnt, unsigned* flags, unsigned target, unsigned epoch) {
     __syncthreads();
+    if (V == 11 || V == 12) {   // counter + broadcast: the last arriver writes every CTA's own go-flag line
+        if (threadIdx.x < 32) {
+            unsigned last = 0;
+            if (threadIdx.x == 0) {
+                __threadfence();
+                unsigned old;
+                asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(cnt), "r"(1u) : "memory");
+                last = (old + 1 == target) ? 1u : 0u;
+            }
+            last = __shfl_sync(0xffffffffu, last, 0);
+            if (last) {
+                for (unsigned c = threadIdx.x; c < gridDim.x; c += 32)
+                    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flags + c * 32), "r"(epoch) : "memory");
+            }
+            if (threadIdx.x == 0) {
+                unsigned v;
+                do {
+                    if (V == 11) asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flags + blockIdx.x * 32) : "memory");
+                    else asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flags + blockIdx.x * 32) : "memory");
+                } while (static_cast<int>(v - epoch) < 0);
+                if (V == 12) asm volatile("fence.acq_rel.gpu;" ::: "memory");
+            }
+        }
+        __syncthreads();
+        return;
+    }
     if (V >= 8) {   // two levels: G sub-counters (own 128-B lines), the last of each group bumps the top
         constexpr int G = V == 8 ? 16 : (V == 9 ? 8 : 32);
         if (threadIdx.x == 0) {
@@ -114,5 +141,6 @@ int main() {
     run<0>(cnt, flags, out); run<1>(cnt, flags, out); run<4>(cnt, flags, out); run<5>(cnt, flags, out);
     run<6>(cnt, flags, out); run<7>(cnt, flags, out); run<0>(cnt, flags, out);
     run<8>(cnt, flags, out); run<9>(cnt, flags, out); run<10>(cnt, flags, out);
+    run<11>(cnt, flags, out); run<12>(cnt, flags, out); run<0>(cnt, flags, out); run<11>(cnt, flags, out);
     return 0;
 }
