@@ -853,7 +853,13 @@ def main():
     if not args.no_sharded:
         props = torch.cuda.get_device_properties(local)
         flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
-        sharded = run_sharded(args, rank, world, local, peaks, flush)
+        if world == 1:
+            try:      # a failing sub-config must not cost the headline line (world 1: no collectives to strand)
+                sharded = run_sharded(args, rank, world, local, peaks, flush)
+            except Exception as e:  # noqa: BLE001
+                sharded = {"error": f"{type(e).__name__}: {e}"}
+        else:
+            sharded = run_sharded(args, rank, world, local, peaks, flush)
         del flush
         if rank == 0:
             line["sharded_configs"] = sharded
@@ -861,7 +867,10 @@ def main():
         if not args.no_extras:
             props = torch.cuda.get_device_properties(local)
             flush = torch.empty(2 * props.L2_cache_size, dtype=torch.uint8, device="cuda")
-            line["configs"] = run_extras(peaks, flush)
+            try:
+                line["configs"] = run_extras(peaks, flush)
+            except Exception as e:  # noqa: BLE001
+                line["configs"] = {"error": f"{type(e).__name__}: {e}"}
             line["configs_timing"] = ("per config: warm-up launches, then each timed launch preceded (outside the "
                                       "CUDA-event pair) by an L2 flush and a ~100-us device sleep so the launch is "
                                       "queued before the start event; median over launches. Flush = write of 2x L2 "
@@ -869,7 +878,10 @@ def main():
                                       "(Black-Scholes map, Mandelbrot, matmul + cuBLAS), else that write followed by "
                                       "a read of another 2x L2 buffer (clean L2): the L2 state the same kernel "
                                       "leaves behind when run back to back")
-            oracle_beside(line["configs"])
+            try:
+                oracle_beside(line["configs"])
+            except Exception as e:  # noqa: BLE001
+                line["configs_oracle_error"] = f"{type(e).__name__}: {e}"
         with one_core():
             v, secs = cpu_oracle_sample(args.n, args.cpu_targets)
         line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
