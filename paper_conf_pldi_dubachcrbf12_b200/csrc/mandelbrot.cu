@@ -243,6 +243,11 @@ cudaError_t launch(int32_t width, int32_t row_first, int32_t row_stride, int32_t
         case 9: return launch_t<4, 32, 16>(a, stream);
         case 10: return launch_t<4, 32, 32>(a, stream);
         case 11: return launch_t<4, 32, 8>(a, stream);
+        case 12: return launch_t<8, 32, 16>(a, stream);     // lazy, 16 x 4 tiles
+        case 13: return launch_t<2, 32, 16>(a, stream);     // lazy, 4 x 16 tiles
+        case 14: return launch_t<4, 32, 12>(a, stream);
+        case 15: return launch_t<4, 32, 24>(a, stream);
+        case 16: return launch_t<4, 32, 20>(a, stream);
         default: return launch_t<4, 32, LIME_MANDEL_LAZY>(a, stream);   // 8x8 tiles, vote every 32 (tools/tune_mandel.py)
     }
 }
