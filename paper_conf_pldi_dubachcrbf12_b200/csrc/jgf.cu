@@ -140,6 +140,13 @@ template <> __device__ __forceinline__ const double* series_sin<double>() { retu
 #define LIME_SERIES_SPLIT 1
 #endif
 constexpr int kSeriesSplit = LIME_SERIES_SPLIT;
+// u-loop unroll (r02 A/B, tools/time_series.py): fp32 1 / 4 / 16 / 64: 21.4 / 20.5 / 19.4 / 27.6 us;
+// fp64 1 / 4 / 16: 31.7 / 36.0 / 42.1 us (register pressure at 4 CTAs/SM) -> 16 for fp32, 1 for fp64
+#ifndef LIME_SERIES_UNROLL_U
+#define LIME_SERIES_UNROLL_U 0
+#endif
+template <typename T>
+constexpr int series_unroll_u() { return LIME_SERIES_UNROLL_U > 0 ? LIME_SERIES_UNROLL_U : (sizeof(T) == 4 ? 16 : 1); }
 template <typename T, int R, int SPLIT>
 __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_kernel(const __grid_constant__ SeriesNodes<T> G,
                                                               int64_t n0, int64_t count, T* __restrict__ out) {
@@ -188,7 +195,8 @@ __global__ void __launch_bounds__(kSeriesBlock, sizeof(T) == 4 ? 8 : 4) series_k
         T gn[R];
 #pragma unroll
         for (int v = 0; v < R; ++v) gn[v] = kAhead ? G.g[h * NUS * R + v] : T(0);
-#pragma unroll 1
+        constexpr int kUnrollU = series_unroll_u<T>();
+#pragma unroll kUnrollU
         for (int u = h * NUS; u < (h + 1) * NUS; ++u) {
             T g[R];
 #pragma unroll
