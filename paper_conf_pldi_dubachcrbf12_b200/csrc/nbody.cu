@@ -94,6 +94,8 @@ struct ForceArgs {
     int chunk;            // chunk_len(n_src)
     int64_t split_len;    // chunks_per_split * chunk
     int tree;             // n_src <= kSmallMaxSources: split partials combined by split_tree_sum
+    int tile_major;       // grid (splits, tiles): a tile's S split CTAs are scheduled back to back,
+                          // so its partials are combined while still in L2 (else grid (tiles, splits))
 };
 
 // Split combine of the small problems (n_src <= kSmallMaxSources): a pairwise tree over
@@ -114,6 +116,14 @@ __device__ __forceinline__ float4 split_tree_sum(int S, Load load) {
     }
     return stack[0];
 }
+
+#ifndef LIME_TILE_MAJOR
+#define LIME_TILE_MAJOR 1
+#endif
+#ifndef LIME_DISCARD_PARTIALS
+#define LIME_DISCARD_PARTIALS 1
+#endif
+static bool nbody_tile_major() { return LIME_TILE_MAJOR != 0; }
 
 template <int R, bool kPacked>
 struct Interact;
@@ -356,6 +366,22 @@ __device__ __forceinline__ void finish_targets(const ForceArgs& a, const IT& it,
         acc.w = 0.f;
         a.accel[t] = acc;
     }
+#if LIME_DISCARD_PARTIALS
+    // The partials are dead once combined: drop their L2 lines without write-back (discard.global.L2),
+    // so with the tile-major grid they never reach DRAM. Only lines wholly inside this tile's slice
+    // of each split row (other tiles' partials may share a boundary line and are still to be read).
+    __syncthreads();                               // every thread has read its partials
+    {
+        const int64_t t0 = tbase, t1 = mn<int64_t>(a.tgt_count, tbase + static_cast<int64_t>(BLOCK) * R);
+        for (int sp = 0; sp < a.splits; ++sp) {
+            const uintptr_t lo = reinterpret_cast<uintptr_t>(a.partial + static_cast<int64_t>(sp) * a.tgt_count + t0);
+            const uintptr_t hi = reinterpret_cast<uintptr_t>(a.partial + static_cast<int64_t>(sp) * a.tgt_count + t1);
+            const uintptr_t l0 = (lo + 127) & ~static_cast<uintptr_t>(127);
+            for (uintptr_t l = l0 + static_cast<uintptr_t>(threadIdx.x) * 128; l + 128 <= hi; l += static_cast<uintptr_t>(BLOCK) * 128)
+                asm volatile("discard.global.L2 [%0], 128;" :: "l"(l) : "memory");
+        }
+    }
+#endif
     if (threadIdx.x == 0) a.counters[tile] = 0u;    // leave the workspace zeroed
 }
 
@@ -365,8 +391,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) force_kernel(const __grid_constan
     __shared__ __align__(8) uint64_t full[2];
     __shared__ int s_last;
 
-    const int tile = blockIdx.x;
-    const int split = blockIdx.y;
+    const int tile = a.tile_major ? blockIdx.y : blockIdx.x;
+    const int split = a.tile_major ? blockIdx.x : blockIdx.y;
     const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * R);
 
     // ---- this split's source range [j0, j1)
@@ -1006,8 +1032,8 @@ __global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_consta
     __shared__ float tx[(V == 4) ? kTileJ : 1], ty[(V == 4) ? kTileJ : 1], tz[(V == 4) ? kTileJ : 1],
         tm[(V == 4) ? kTileJ : 1];
     __shared__ int s_last;
-    const int tile = blockIdx.x;
-    const int split = blockIdx.y;
+    const int tile = a.tile_major ? blockIdx.y : blockIdx.x;
+    const int split = a.tile_major ? blockIdx.x : blockIdx.y;
     const int64_t tbase = static_cast<int64_t>(tile) * (BLOCK * R);
     Interact<R, kPacked> it;
     bool valid[R];
@@ -1078,19 +1104,22 @@ __global__ void __launch_bounds__(BLOCK) force_ablate_kernel(const __grid_consta
 template <int BLOCK, int R>
 static cudaError_t launch_ablate(const ForceArgs& a, int v, cudaStream_t stream) {
     const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
-    dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
+    ForceArgs b = a;
+    b.tile_major = tiles <= 65535 && nbody_tile_major();
+    const dim3 grid = b.tile_major ? dim3(static_cast<unsigned>(b.splits), static_cast<unsigned>(tiles))
+                                   : dim3(static_cast<unsigned>(tiles), static_cast<unsigned>(b.splits));
     switch (v) {
-        case 1: force_ablate_kernel<BLOCK, R, 1><<<grid, BLOCK, 0, stream>>>(a); break;
-        case 2: force_ablate_kernel<BLOCK, R, 2><<<grid, BLOCK, 0, stream>>>(a); break;
-        case 3: force_ablate_kernel<BLOCK, R, 3><<<grid, BLOCK, 0, stream>>>(a); break;
-        case 4: force_ablate_kernel<BLOCK, R, 4><<<grid, BLOCK, 0, stream>>>(a); break;
-        case 5: force_ablate_kernel<BLOCK, R, 5><<<grid, BLOCK, 0, stream>>>(a); break;
+        case 1: force_ablate_kernel<BLOCK, R, 1><<<grid, BLOCK, 0, stream>>>(b); break;
+        case 2: force_ablate_kernel<BLOCK, R, 2><<<grid, BLOCK, 0, stream>>>(b); break;
+        case 3: force_ablate_kernel<BLOCK, R, 3><<<grid, BLOCK, 0, stream>>>(b); break;
+        case 4: force_ablate_kernel<BLOCK, R, 4><<<grid, BLOCK, 0, stream>>>(b); break;
+        case 5: force_ablate_kernel<BLOCK, R, 5><<<grid, BLOCK, 0, stream>>>(b); break;
         case 6: {
             if (a.n_src > kConstBodies) return cudaErrorInvalidValue;
             cudaError_t e = cudaMemcpyToSymbolAsync(c_bodies, a.bodies, static_cast<size_t>(a.n_src) * 16, 0,
                                                     cudaMemcpyDeviceToDevice, stream);
             if (e != cudaSuccess) return e;
-            force_ablate_kernel<BLOCK, R, 6><<<grid, BLOCK, 0, stream>>>(a);
+            force_ablate_kernel<BLOCK, R, 6><<<grid, BLOCK, 0, stream>>>(b);
             break;
         }
         default: return cudaErrorInvalidValue;
@@ -1105,13 +1134,16 @@ static cudaError_t launch_one(const ForceArgs& a, cudaStream_t stream) {
     constexpr bool kPacked = (R % 2 == 0);
     constexpr int MINB = BLOCK == 512 ? 1 : 0;
     const int64_t tiles = ceil_div<int64_t>(a.tgt_count, static_cast<int64_t>(BLOCK) * R);
-    dim3 grid(static_cast<unsigned>(tiles), static_cast<unsigned>(a.splits));
-    if (a.chunk == kChunk) {
+    ForceArgs b = a;
+    b.tile_major = tiles <= 65535 && nbody_tile_major();
+    const dim3 grid = b.tile_major ? dim3(static_cast<unsigned>(b.splits), static_cast<unsigned>(tiles))
+                                   : dim3(static_cast<unsigned>(tiles), static_cast<unsigned>(b.splits));
+    if (b.chunk == kChunk) {
         // mass-uniform splits, then the others (each CTA of either launch leaves unless its split is its kind)
-        if (a.uniform != nullptr) force_kernel<BLOCK, R, kPacked, kChunk, MINB, true><<<grid, BLOCK, 0, stream>>>(a);
-        force_kernel<BLOCK, R, kPacked, kChunk, MINB><<<grid, BLOCK, 0, stream>>>(a);
+        if (b.uniform != nullptr) force_kernel<BLOCK, R, kPacked, kChunk, MINB, true><<<grid, BLOCK, 0, stream>>>(b);
+        force_kernel<BLOCK, R, kPacked, kChunk, MINB><<<grid, BLOCK, 0, stream>>>(b);
     } else {
-        force_kernel<BLOCK, R, kPacked, kChunkSmall, MINB><<<grid, BLOCK, 0, stream>>>(a);
+        force_kernel<BLOCK, R, kPacked, kChunkSmall, MINB><<<grid, BLOCK, 0, stream>>>(b);
     }
     return cudaGetLastError();
 }
@@ -1130,6 +1162,7 @@ cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin,
     a.chunk = chunk_len(n_src);
     a.split_len = chunks_per_split(n_src) * a.chunk;
     a.tree = n_src <= kSmallMaxSources;
+    a.tile_major = 0;
     a.counters = static_cast<unsigned*>(ws);
     a.uniform = nullptr;
     a.partial = reinterpret_cast<float4*>(static_cast<char*>(ws) + counters_bytes(tgt_count) + flags_bytes(n_src));
