@@ -21,6 +21,10 @@
 #include "common.cuh"
 #include "kernels.h"
 
+#ifndef LIME_GEMM_SNAKE
+#define LIME_GEMM_SNAKE 1
+#endif
+
 namespace lime {
 namespace gemm {
 
@@ -102,6 +106,11 @@ __device__ __forceinline__ void tile_coords(int t, const Params& p, int& mb, int
     const int r = t - g * per_group;
     mb = first_m + r % gm;
     nb = r / gm;
+#if LIME_GEMM_SNAKE
+    // serpentine sweep: odd groups walk the N tiles backwards, so the Bt tiles the previous group
+    // touched last -- still in L2 -- are the first ones this group reads
+    if (g & 1) nb = p.num_n - 1 - nb;
+#endif
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
@@ -311,6 +320,11 @@ __device__ __forceinline__ void tile_coords2(int t, const Params2& p, int& mb, i
     const int r = t - g * per_group;
     mb = first_m + r % gm;
     nb = r / gm;
+#if LIME_GEMM_SNAKE
+    // serpentine sweep: odd groups walk the N tiles backwards, so the Bt tiles the previous group
+    // touched last -- still in L2 -- are the first ones this group reads
+    if (g & 1) nb = p.num_n - 1 - nb;
+#endif
 }
 
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
