@@ -504,19 +504,31 @@ constexpr int kSmallMaxThreads = LIME_SMALL_MAXT;   // block cap (register budge
 constexpr size_t kOneCtaPerSmSmem = 116 * 1024;   // > 228 KB / 2 per SM (B200)
 
 // One split's contribution for the lane's targets: chunk partials added into the split accumulator
-// in chunk order -- the arithmetic of force_kernel.
+// in chunk order -- the arithmetic of force_kernel. Chunks flagged in umask (bit c: chunk c of the
+// split; simulate_small_kernel only, see small_unit_flags) take the factored form, which rounds
+// exactly like the per-body form for their masses.
 template <class IT>
-__device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2) {
-    for (int c0 = 0; c0 < len; c0 += chunk) {
+__device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2, uint32_t umask) {
+    for (int c0 = 0, c = 0; c0 < len; c0 += chunk, ++c) {
         const int c1 = mn(len, c0 + chunk);
         it.chunk_begin();
-        if (c1 - c0 == kChunkSmall) {
+        if ((umask >> c) & 1u) {
+            if (c1 - c0 == kChunkSmall) {
 #pragma unroll kSmallUnroll
-            for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
+                for (int j = c0; j < c0 + kChunkSmall; ++j) it.body_unit(sb[j], eps2);
+            } else {
+                for (int j = c0; j < c1; ++j) it.body_unit(sb[j], eps2);
+            }
+            it.chunk_end_scaled(sb[c0].w);
         } else {
-            for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+            if (c1 - c0 == kChunkSmall) {
+#pragma unroll kSmallUnroll
+                for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
+            } else {
+                for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+            }
+            it.chunk_end();
         }
-        it.chunk_end();
     }
 }
 
@@ -622,14 +634,21 @@ __device__ int g_lime_step;
 // Lane -> work map shared by both small kernels.
 struct SmallLane {
     int gslot, s, p;   // group slot in this CTA, split, pair within the group
-    __device__ __forceinline__ SmallLane(int S2) {
-        const int idx = static_cast<int>(threadIdx.x) % (kGroupPairs * S2);
-        gslot = static_cast<int>(threadIdx.x) / (kGroupPairs * S2);
+    __device__ __forceinline__ SmallLane(int S2) {              // kGroupPairs * S2: a power of two
+        const int lg = __ffs(kGroupPairs * S2) - 1;
+        const int idx = static_cast<int>(threadIdx.x) & ((1 << lg) - 1);
+        gslot = static_cast<int>(threadIdx.x) >> lg;
         s = idx / kGroupPairs;
         p = idx % kGroupPairs;
     }
 };
-__device__ __forceinline__ int padded(int i, int L) { return (i / L) * (L + 1) + i % L; }
+// The small path's split length L is 64 or 128 (a power of two: at most 2 x 64 chunks of 64 bodies
+// over 64 splits), so the padded slot i + i / L is a shift -- a runtime integer division costs ~20
+// instructions, and every warp of the 4096-body kernel did ~10 of them before its loop.
+static_assert(kSmallMaxSources / kChunkSmall <= 2 * kMaxSplitsSmall, "split length 64 or 128 (a power of two)");
+__device__ __forceinline__ int lg2i(int L) { return __ffs(L) - 1; }
+__device__ __forceinline__ int split_of(int i, int L) { return i >> lg2i(L); }
+__device__ __forceinline__ int padded(int i, int L) { return i + split_of(i, L); }
 
 #ifndef LIME_STAGE_U
 #define LIME_STAGE_U 6
@@ -656,13 +675,72 @@ __device__ __forceinline__ void stage_all(float4* src, const float4* bodies, int
     }
 }
 
+// Persistent simulation only (R11 at the small sizes): a 64-body chunk whose masses all equal one
+// power of two m = 2^e, -40 <= e <= 20, is summed in the factored form -- sum_j d_j / R_j^3, scaled
+// by m once (11 FP32 lane-ops per interaction instead of 12). Scaling by a power of two is exact,
+// so each factored product and partial is exactly m times its per-body counterpart and the result
+// has the per-body form's bits whenever no intermediate is subnormal or infinite (eps^2 >= 1e-20
+// is required, which bounds R^-3 by 1e30; coordinates up to ~1e6 keep m R^-3 |d| normal); the
+// other kernels need no decision and the simulation stays bit-identical to eager steps. Masses never change
+// during a simulation, so the whole CTA finds the flags once, in step 0, from global memory: one
+// per 32-body half chunk (body i against the first mass of its chunk; bodies past n count as
+// equal). Per launch this costs more than it saves (measured: +1.2-2 us per 4096-body force
+// launch for ~1.2 us of FP32 work), so the one-step kernels keep the per-body form.
+#ifndef LIME_SIM_FACTOR
+#define LIME_SIM_FACTOR 1
+#endif
+constexpr int kMaxHalfChunks = 2 * static_cast<int>(kSmallMaxSources / kChunkSmall);
+static_assert(kChunkSmall == 64, "half chunks are one warp wide");
+__device__ __forceinline__ bool unit_mass(float m) {
+    const uint32_t b = __float_as_uint(m);
+    return (b & 0x807fffffu) == 0u && (b >> 23) >= 127u - 40u && (b >> 23) <= 127u + 20u;   // +2^e, -40 <= e <= 20
+}
+__device__ __forceinline__ void small_unit_flags(const float4* bodies, int64_t n, uint8_t* hflags) {
+    constexpr int U = 8;                               // loads in flight per lane (4096 bodies: 5 per lane)
+    const int nh = static_cast<int>(ceil_div<int64_t>(n, 32));
+    const int nw = static_cast<int>(blockDim.x >> 5), w = static_cast<int>(threadIdx.x >> 5);
+    const float* mass = reinterpret_cast<const float*>(bodies) + 3;
+    for (int h0 = w; h0 < nh; h0 += U * nw) {
+        float m[U], m0[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int h = h0 + u * nw, i = h * 32 + static_cast<int>(lane_id());
+            m[u] = m0[u] = 0.f;
+            if (h < nh) {
+                m0[u] = __ldcg(mass + 4 * ((h >> 1) * kChunkSmall));
+                m[u] = i < n ? __ldcg(mass + 4 * i) : m0[u];
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int h = h0 + u * nw;
+            const bool uni = __all_sync(0xffffffffu, m[u] == m0[u]) && unit_mass(m0[u]);
+            if (h < nh && lane_id() == 0) hflags[h] = uni ? 1 : 0;
+        }
+    }
+}
+// Bit c: chunk c of split s is mass-uniform (both its half chunks flagged).
+__device__ __forceinline__ uint32_t lane_unit_mask(const uint8_t* hflags, int s, int S, int L, int64_t n) {
+    uint32_t mask = 0;
+    if (s >= S) return 0;
+    const int nh = static_cast<int>(ceil_div<int64_t>(n, 32));
+    for (int c = 0; c < L / kChunkSmall; ++c) {
+        const int h = 2 * (s * (L / kChunkSmall) + c);
+        if (h >= nh) break;
+        const bool uni = hflags[h] != 0 && (h + 1 >= nh || hflags[h + 1] != 0);
+        mask |= static_cast<uint32_t>(uni) << c;
+    }
+    return mask;
+}
+
 // The lane's split partial for targets tg + 2p, tg + 2p + 1 (clamped to the last valid target),
 // then the butterfly over the warp's splits: lanes 2 (16 w) + p of each group's warp w end up with
 // the sum of splits 16 w .. 16 w + 15 (or the whole group when S2 <= 16), stored to wpart.
 // Every lane of the CTA's used warps calls it (lanes of split s >= S contribute zero).
 __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLane& sl, bool active, int64_t tgt_first_src,
                                                int64_t tg, int64_t tcount, int L, int S, int S2, int64_t n, int chunk,
-                                               float eps2, float4* wpart, uint64_t* tbar, uint32_t parity) {
+                                               float eps2, float4* wpart, uint64_t* tbar, uint32_t parity,
+                                               uint32_t umask) {
     Interact<2, true> it;
     it.zero_all();
     LIME_WTRACE(0);
@@ -672,7 +750,7 @@ __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLan
             int64_t t = tg + 2 * sl.p + r;
             t = t < tcount ? t : tcount - 1;
             const int i = static_cast<int>(tgt_first_src + t);
-            if (tbar) mbar_wait(&tbar[(i / L) / kStageRows], parity);
+            if (tbar) mbar_wait(&tbar[split_of(i, L) / kStageRows], parity);
             it.set(r, src[padded(i, L)]);
         }
         if (tbar) mbar_wait(&tbar[sl.s / kStageRows], parity);
@@ -683,7 +761,7 @@ __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLan
     if (active && sl.s < S) {
         const int64_t j0 = static_cast<int64_t>(sl.s) * L;
         split_sum(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
-                  eps2);
+                  eps2, umask);
     }
     float4 a0 = it.result(0), a1 = it.result(1);
     const int seg = S2 < kWarpSplits ? kGroupPairs * S2 : 32;   // lanes of one group within this warp
@@ -754,7 +832,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
     for (int64_t r0 = gb; r0 < ge; r0 += slots) {
         const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
         small_lane_sum(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
-                       a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0);
+                       a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0, 0u);
         __syncthreads();
         const int64_t t = r0 * kGroupTargets + ct;
         if (ct < ng * kGroupTargets && t < a.tgt_count) {
@@ -763,7 +841,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
                 a.accel[t] = acc;
             } else {                                   // integrate_kernel's arithmetic on the old position
                 const int i = static_cast<int>(a.tgt_begin + t);
-                if (a.tma) mbar_wait(&tbar[(i / a.L) / kStageRows], 0);
+                if (a.tma) mbar_wait(&tbar[split_of(i, a.L) / kStageRows], 0);
                 float4 p = src[padded(i, a.L)];
                 float4 v = a.vel[t];
                 v.x = fmaf(acc.x, a.dt, v.x);
@@ -833,6 +911,7 @@ struct SimArgs {
     int64_t groups;
     float eps2, dt;
     int tma, rows;
+    int factor;          // eps2 >= 1e-20: factored mass-uniform chunks allowed (see small_unit_flags)
 };
 
 __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target) {
@@ -856,6 +935,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
     float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
     float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.rows, a.L));   // [slots][blocks][4]
     __shared__ __align__(8) uint64_t tbar[kMaxStageCopies];
+    __shared__ uint8_t hflags[kMaxHalfChunks];
     if (a.tma) {
         if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) mbar_init(&tbar[threadIdx.x], 1);
         fence_mbar_init();
@@ -867,6 +947,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
     const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
     const int ct = static_cast<int>(threadIdx.x);      // combine thread: one target of the round's groups
     unsigned barrier_target = 0;
+    uint32_t umask = 0;                                // the lane's factored chunks (masses never change: step 0)
 
     for (int32_t k = 0; k < a.steps; ++k) {
         const float4* cur = (k & 1) ? a.pos_alt : a.pos;
@@ -886,6 +967,11 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             stage_all<true>(src, cur, a.n, a.L);   // what every CTA wrote in the previous step (L2)
             __syncthreads();
         }
+        if (k == 0) {
+            small_unit_flags(a.pos, a.n, hflags);      // step 0 reads pos: nothing has written it yet
+            __syncthreads();
+            umask = a.factor ? lane_unit_mask(hflags, sl.s, a.S, a.L, a.n) : 0u;
+        }
         LIME_TRACE_AT(k, 6);
         for (int64_t r0 = gb; r0 < ge; r0 += slots) {
             const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
@@ -894,13 +980,13 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
             if (owner) v = a.vel[t];                   // issued before the force work: latency hidden
             small_lane_sum(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
-                           a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1));
+                           a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1), umask);
             LIME_TRACE_AT(k, 4);
             __syncthreads();
             LIME_TRACE_AT(k, 1);
             if (owner) {
                 const float4 acc = small_target_sum(wpart, ct, a.S2);
-                if (a.tma) mbar_wait(&tbar[(static_cast<int>(t) / a.L) / kStageRows], static_cast<uint32_t>(k & 1));
+                if (a.tma) mbar_wait(&tbar[split_of(static_cast<int>(t), a.L) / kStageRows], static_cast<uint32_t>(k & 1));
                 float4 pn = src[padded(static_cast<int>(t), a.L)];
                 v.x = fmaf(acc.x, a.dt, v.x);
                 v.y = fmaf(acc.y, a.dt, v.y);
@@ -987,6 +1073,7 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.dt = dt;
     a.tma = p.tma;
     a.rows = p.rows;
+    a.factor = (eps2 >= 1e-20f && LIME_SIM_FACTOR) ? 1 : 0;
     CUtensorMap map_pos, map_alt;
     std::memset(&map_pos, 0, sizeof map_pos);
     std::memset(&map_alt, 0, sizeof map_alt);

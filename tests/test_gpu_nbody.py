@@ -379,3 +379,53 @@ def test_tma_staged_sizes_match_general_kernel(lime, n):
     pe, ve = b.clone(), torch.zeros_like(b)
     _eager_steps(lime, pe, ve, 3)
     assert torch.equal(pos, pe) and torch.equal(vel, ve)
+
+
+# ------------------------------ R11 at the small sizes: factored power-of-two chunks (persistent simulation)
+def _mixed_chunk_bodies(n, seed):
+    """Chunk 0 (and every chunk not listed) mass 2^-12; chunk 1 random masses; chunk 2 one body off
+    by one ulp; chunk 3 massless; chunk 4 equal but not a power of two (1/3000); chunk 5 equal 2^-41
+    (outside the factored range); the ragged last chunk 2^3."""
+    b = inputs.nbody_bodies(n, seed=seed)
+    b[:, 3] = np.float32(2.0 ** -12)
+    rng = np.random.default_rng(seed)
+    b[64:128, 3] = rng.uniform(1e-4, 1e-3, 64).astype(np.float32)
+    b[128 + 17, 3] = np.nextafter(b[128 + 17, 3], np.float32(1))
+    b[192:256, 3] = 0.0
+    b[256:320, 3] = np.float32(1.0 / 3000)
+    b[320:384, 3] = np.float32(2.0 ** -41)
+    tail = n - (n % 64 or 64)
+    b[tail:, 3] = np.float32(8.0)
+    return b
+
+
+@pytest.mark.parametrize("n", [400, 4096, 4160, 5000, 8192])
+def test_simulate_factored_chunks_bit_identical(lime, n):
+    # simulate_small_kernel sums chunks of equal power-of-two masses in the factored (11-op) form;
+    # scaling by a power of two is exact, so it must still equal eager per-body steps bit for bit,
+    # and the oracle within tolerance
+    b_np = _mixed_chunk_bodies(n, 400 + n)
+    b = _dev(b_np)
+    v0 = (inputs.nbody_bodies(n, seed=401 + n) * np.float32(0.05)).astype(np.float32)
+    v0[:, 3] = 0
+    pos, vel = b.clone(), _dev(v0)
+    lime.nbody_simulate(pos, vel, 4, float(EPS2), 1e-3)
+    pe, ve = b.clone(), _dev(v0)
+    _eager_steps(lime, pe, ve, 4)
+    assert torch.equal(pos, pe) and torch.equal(vel, ve)
+    # one step from rest against the oracle: v1 = a dt (dt = 2^-10, exact scaling)
+    p1, v1 = b.clone(), torch.zeros_like(b)
+    lime.nbody_simulate(p1, v1, 1, float(EPS2), 2.0 ** -10)
+    ref, mag = oracle.nbody_accel(b_np, EPS2, with_mag=True)
+    assert nbody_rel_err(v1.cpu().numpy() * 1024.0, ref, mag).max() <= NBODY_RTOL
+
+
+def test_simulate_factored_needs_softening(lime):
+    # eps^2 < 1e-20 turns the factored form off (it bounds R^-3); still bit-identical
+    n = 4096
+    b = _dev(_mixed_chunk_bodies(n, 9))
+    pos, vel = b.clone(), torch.zeros_like(b)
+    lime.nbody_simulate(pos, vel, 2, 1e-22, 1e-3)
+    pe, ve = b.clone(), torch.zeros_like(b)
+    _eager_steps(lime, pe, ve, 2, eps2=1e-22)
+    assert torch.equal(pos, pe) and torch.equal(vel, ve)
