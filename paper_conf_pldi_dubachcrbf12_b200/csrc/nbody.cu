@@ -38,11 +38,18 @@ namespace nbody {
 #define LIME_BODY_UNROLL 4
 #endif
 constexpr int kUnitUnroll = LIME_UNIT_UNROLL;
+// Small-kernel inner loop unroll (sources), per kernel -- r02 A/B (tools/ab_small_nbody.py, 4096
+// bodies, graph / persistent us per step): 4: 10.69 / 10.55, 8: 10.53 / 10.39, 16: 10.73 / 10.29,
+// 64 (the whole chunk): 10.39 / 10.41 (profiles/experiments/small_nbody_unroll_r02.json)
 #ifndef LIME_SMALL_UNROLL
-#define LIME_SMALL_UNROLL 8            // r01t A/B: 4096-body graph / persistent step 12.10 -> 11.85 us (2 is slower)
+#define LIME_SMALL_UNROLL 64           // force_small_kernel (one-step map / fused step)
+#endif
+#ifndef LIME_SIM_UNROLL
+#define LIME_SIM_UNROLL 16             // simulate_small_kernel
 #endif
 constexpr int kBodyUnroll = LIME_BODY_UNROLL;
 constexpr int kSmallUnroll = LIME_SMALL_UNROLL;
+constexpr int kSimUnroll = LIME_SIM_UNROLL;
 constexpr int kTileJ = 1024;   // sources per shared-memory stage (16 KB)
 static_assert(kTileJ % kChunk == 0 && kTileJ % kChunkSmall == 0, "stage must hold whole chunks");
 
@@ -507,14 +514,14 @@ constexpr size_t kOneCtaPerSmSmem = 116 * 1024;   // > 228 KB / 2 per SM (B200)
 // in chunk order -- the arithmetic of force_kernel. Chunks flagged in umask (bit c: chunk c of the
 // split; simulate_small_kernel only, see small_unit_flags) take the factored form, which rounds
 // exactly like the per-body form for their masses.
-template <class IT>
+template <int U, class IT>
 __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2, uint32_t umask) {
     for (int c0 = 0, c = 0; c0 < len; c0 += chunk, ++c) {
         const int c1 = mn(len, c0 + chunk);
         it.chunk_begin();
         if ((umask >> c) & 1u) {
             if (c1 - c0 == kChunkSmall) {
-#pragma unroll kSmallUnroll
+#pragma unroll U
                 for (int j = c0; j < c0 + kChunkSmall; ++j) it.body_unit(sb[j], eps2);
             } else {
                 for (int j = c0; j < c1; ++j) it.body_unit(sb[j], eps2);
@@ -522,7 +529,7 @@ __device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int
             it.chunk_end_scaled(sb[c0].w);
         } else {
             if (c1 - c0 == kChunkSmall) {
-#pragma unroll kSmallUnroll
+#pragma unroll U
                 for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
             } else {
                 for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
@@ -737,6 +744,7 @@ __device__ __forceinline__ uint32_t lane_unit_mask(const uint8_t* hflags, int s,
 // then the butterfly over the warp's splits: lanes 2 (16 w) + p of each group's warp w end up with
 // the sum of splits 16 w .. 16 w + 15 (or the whole group when S2 <= 16), stored to wpart.
 // Every lane of the CTA's used warps calls it (lanes of split s >= S contribute zero).
+template <int U>
 __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLane& sl, bool active, int64_t tgt_first_src,
                                                int64_t tg, int64_t tcount, int L, int S, int S2, int64_t n, int chunk,
                                                float eps2, float4* wpart, uint64_t* tbar, uint32_t parity,
@@ -760,7 +768,7 @@ __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLan
     __syncwarp();
     if (active && sl.s < S) {
         const int64_t j0 = static_cast<int64_t>(sl.s) * L;
-        split_sum(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
+        split_sum<U>(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
                   eps2, umask);
     }
     float4 a0 = it.result(0), a1 = it.result(1);
@@ -831,7 +839,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
     // take part in its butterfly), lanes beyond the round's groups inactive
     for (int64_t r0 = gb; r0 < ge; r0 += slots) {
         const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
-        small_lane_sum(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
+        small_lane_sum<kSmallUnroll>(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
                        a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0, 0u);
         __syncthreads();
         const int64_t t = r0 * kGroupTargets + ct;
@@ -979,7 +987,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             const bool owner = ct < ng * kGroupTargets && t < a.n;
             float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
             if (owner) v = a.vel[t];                   // issued before the force work: latency hidden
-            small_lane_sum(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
+            small_lane_sum<kSimUnroll>(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
                            a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1), umask);
             LIME_TRACE_AT(k, 4);
             __syncthreads();
