@@ -588,7 +588,9 @@ struct SmallPlan {
     int block;           // slots x 2 S2 lanes, rounded up to whole warps
     size_t smem;
 };
-__host__ __device__ __forceinline__ int64_t group_begin(int64_t groups, int grid, int c) { return groups * c / grid; }
+// CTA c's groups: [c q + min(c, r), + q + (c < r)) with q = groups / grid, r = groups % grid taken
+// on the host (a runtime division per thread costs ~20 SASS instructions).
+__device__ __forceinline__ int group_begin(int q, int r, int c) { return c * q + mn(c, r); }
 __host__ __device__ __forceinline__ int warp_blocks(int S2) { return S2 > kWarpSplits ? S2 / kWarpSplits : 1; }
 __host__ __device__ __forceinline__ size_t small_src_bytes(int S, int L) { return static_cast<size_t>(S) * (L + 1) * 16; }
 
@@ -806,6 +808,7 @@ struct SmallArgs {
     float4* accel;
     int S, S2, L, chunk;
     int64_t groups;
+    int gq, gr;          // groups / grid, groups % grid (group_begin)
     int tma;             // sources staged by TMA row boxes (map), else LDG
     int rows;
     // fused step (lime_map_nbody_step): integrate the targets instead of storing accel
@@ -821,8 +824,8 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
     float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.rows, a.L));   // [slots][blocks][4]
     __shared__ __align__(8) uint64_t tbar[kMaxStageCopies];
     pdl_enter();
-    const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
-    const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
+    const int64_t gb = group_begin(a.gq, a.gr, static_cast<int>(blockIdx.x));
+    const int64_t ge = group_begin(a.gq, a.gr, static_cast<int>(blockIdx.x) + 1);
     if (a.tma) {
         if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) mbar_init(&tbar[threadIdx.x], 1);
         fence_mbar_init();
@@ -833,7 +836,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
         __syncthreads();
     }
     const SmallLane sl(a.S2);
-    const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
+    const int slots = static_cast<int>(blockDim.x) >> (__ffs(kGroupPairs * a.S2) - 1);   // a power of two
     const int ct = static_cast<int>(threadIdx.x);
     // rounds of `slots` groups (one round by default); every lane calls small_lane_sum (whole warps
     // take part in its butterfly), lanes beyond the round's groups inactive
@@ -883,6 +886,8 @@ static cudaError_t launch_small(const ForceArgs& f, cudaStream_t stream, float4*
     a.L = p.L;
     a.chunk = p.chunk;
     a.groups = p.groups;
+    a.gq = static_cast<int>(p.groups / p.grid);
+    a.gr = static_cast<int>(p.groups % p.grid);
     a.tma = p.tma;
     a.rows = p.rows;
     a.vel = vel;
@@ -917,6 +922,7 @@ struct SimArgs {
     int32_t steps;
     int32_t S, S2, L, chunk;
     int64_t groups;
+    int gq, gr;          // groups / grid, groups % grid (group_begin)
     float eps2, dt;
     int tma, rows;
     int factor;          // eps2 >= 1e-20: factored mass-uniform chunks allowed (see small_unit_flags)
@@ -949,10 +955,10 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
         fence_mbar_init();
         __syncthreads();
     }
-    const int64_t gb = group_begin(a.groups, gridDim.x, blockIdx.x);
-    const int64_t ge = group_begin(a.groups, gridDim.x, blockIdx.x + 1);
+    const int64_t gb = group_begin(a.gq, a.gr, static_cast<int>(blockIdx.x));
+    const int64_t ge = group_begin(a.gq, a.gr, static_cast<int>(blockIdx.x) + 1);
     const SmallLane sl(a.S2);
-    const int slots = static_cast<int>(blockDim.x) / (kGroupPairs * a.S2);
+    const int slots = static_cast<int>(blockDim.x) >> (__ffs(kGroupPairs * a.S2) - 1);   // a power of two
     const int ct = static_cast<int>(threadIdx.x);      // combine thread: one target of the round's groups
     unsigned barrier_target = 0;
     uint32_t umask = 0;                                // the lane's factored chunks (masses never change: step 0)
@@ -1077,6 +1083,8 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.L = p.L;
     a.chunk = p.chunk;
     a.groups = p.groups;
+    a.gq = static_cast<int>(p.groups / p.grid);
+    a.gr = static_cast<int>(p.groups % p.grid);
     a.eps2 = eps2;
     a.dt = dt;
     a.tma = p.tma;
