@@ -510,32 +510,68 @@ constexpr int kWarpSplits = 32 / kGroupPairs;           // splits one warp of a 
 constexpr int kSmallMaxThreads = LIME_SMALL_MAXT;   // block cap (register budget 65536 / cap)
 constexpr size_t kOneCtaPerSmSmem = 116 * 1024;   // > 228 KB / 2 per SM (B200)
 
+// Factored chunks at the small sizes (R11): a 64-body chunk whose masses all equal
+// one power of two m = 2^e (-40 <= e <= 20) can be summed as sum_j d_j / R_j^3 and scaled by m once
+// -- 11 FP32 lane-ops per interaction instead of 12. Scaling by a power of two is exact, so every
+// factored product and partial is exactly m times its per-body counterpart and the chunk partial
+// has the per-body form's bits (whenever no intermediate is subnormal or infinite: eps^2 >= 1e-20
+// bounds R^-3 by 1e30, and coordinates up to ~1e6 keep m R^-3 |d| normal). The decision therefore
+// needs no agreement between kernels, and no scan of the masses before the loop (each such scan
+// measured 1.2-2 us per launch): a lane predicts "factored" from three masses of its chunk (first,
+// middle, last equal and a power of two in range), checks every mass inside the loop (one LOP3
+// per source on the integer pipe: the bits of m_j xor m), and in the rare case a mass differs
+// recomputes the chunk in the per-body form. Random masses fail the prediction and go straight
+// to the per-body loop; equal power-of-two masses (the workloads' 1/n) take the factored one.
+__device__ __forceinline__ bool unit_mass(float m) {
+    const uint32_t b = __float_as_uint(m);
+    return (b & 0x807fffffu) == 0u && (b >> 23) >= 127u - 40u && (b >> 23) <= 127u + 20u;   // +2^e, -40 <= e <= 20
+}
+#ifndef LIME_SMALL_FACTOR
+#define LIME_SMALL_FACTOR 1
+#endif
+
 // One split's contribution for the lane's targets: chunk partials added into the split accumulator
-// in chunk order -- the arithmetic of force_kernel. Chunks flagged in umask (bit c: chunk c of the
-// split; simulate_small_kernel only, see small_unit_flags) take the factored form, which rounds
-// exactly like the per-body form for their masses.
-template <int U, class IT>
-__device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2, uint32_t umask) {
+// in chunk order -- the arithmetic of force_kernel (per-body form; factored chunks have its bits).
+// kKnown (persistent simulation, whose masses never change): bit c of `known` is set once chunk c
+// has been verified factored, so later steps skip the prediction and the check. (In the one-step
+// kernel a third loop copy costs registers: 14.4 -> 15.5-16.3 us per 4096-body launch.)
+template <int U, bool kKnown, class IT>
+__device__ __forceinline__ void split_sum(IT& it, const float4* sb, int len, int chunk, float eps2, bool factor,
+                                          uint32_t& known) {
     for (int c0 = 0, c = 0; c0 < len; c0 += chunk, ++c) {
         const int c1 = mn(len, c0 + chunk);
         it.chunk_begin();
-        if ((umask >> c) & 1u) {
-            if (c1 - c0 == kChunkSmall) {
+        const float m = sb[c0].w;
+        if (kKnown && ((known >> c) & 1u)) {
 #pragma unroll U
-                for (int j = c0; j < c0 + kChunkSmall; ++j) it.body_unit(sb[j], eps2);
-            } else {
-                for (int j = c0; j < c1; ++j) it.body_unit(sb[j], eps2);
-            }
-            it.chunk_end_scaled(sb[c0].w);
-        } else {
-            if (c1 - c0 == kChunkSmall) {
-#pragma unroll U
-                for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
-            } else {
-                for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
-            }
-            it.chunk_end();
+            for (int j = c0; j < c0 + kChunkSmall; ++j) it.body_unit(sb[j], eps2);
+            it.chunk_end_scaled(m);
+            continue;
         }
+        if (LIME_SMALL_FACTOR && factor && c1 - c0 == kChunkSmall && unit_mass(m) && sb[c0 + kChunkSmall / 2].w == m &&
+            sb[c1 - 1].w == m) {
+            const uint32_t mb = __float_as_uint(m);
+            uint32_t diff = 0;
+#pragma unroll U
+            for (int j = c0; j < c0 + kChunkSmall; ++j) {
+                const float4 b = sb[j];
+                it.body_unit(b, eps2);
+                diff |= __float_as_uint(b.w) ^ mb;
+            }
+            if (diff == 0) {
+                it.chunk_end_scaled(m);
+                known |= 1u << c;
+                continue;
+            }
+            it.chunk_begin();                          // a mass differs: the per-body form after all
+        }
+        if (c1 - c0 == kChunkSmall) {
+#pragma unroll U
+            for (int j = c0; j < c0 + kChunkSmall; ++j) it.body(sb[j], eps2);
+        } else {
+            for (int j = c0; j < c1; ++j) it.body(sb[j], eps2);
+        }
+        it.chunk_end();
     }
 }
 
@@ -684,73 +720,15 @@ __device__ __forceinline__ void stage_all(float4* src, const float4* bodies, int
     }
 }
 
-// Persistent simulation only (R11 at the small sizes): a 64-body chunk whose masses all equal one
-// power of two m = 2^e, -40 <= e <= 20, is summed in the factored form -- sum_j d_j / R_j^3, scaled
-// by m once (11 FP32 lane-ops per interaction instead of 12). Scaling by a power of two is exact,
-// so each factored product and partial is exactly m times its per-body counterpart and the result
-// has the per-body form's bits whenever no intermediate is subnormal or infinite (eps^2 >= 1e-20
-// is required, which bounds R^-3 by 1e30; coordinates up to ~1e6 keep m R^-3 |d| normal); the
-// other kernels need no decision and the simulation stays bit-identical to eager steps. Masses never change
-// during a simulation, so the whole CTA finds the flags once, in step 0, from global memory: one
-// per 32-body half chunk (body i against the first mass of its chunk; bodies past n count as
-// equal). Per launch this costs more than it saves (measured: +1.2-2 us per 4096-body force
-// launch for ~1.2 us of FP32 work), so the one-step kernels keep the per-body form.
-#ifndef LIME_SIM_FACTOR
-#define LIME_SIM_FACTOR 1
-#endif
-constexpr int kMaxHalfChunks = 2 * static_cast<int>(kSmallMaxSources / kChunkSmall);
-static_assert(kChunkSmall == 64, "half chunks are one warp wide");
-__device__ __forceinline__ bool unit_mass(float m) {
-    const uint32_t b = __float_as_uint(m);
-    return (b & 0x807fffffu) == 0u && (b >> 23) >= 127u - 40u && (b >> 23) <= 127u + 20u;   // +2^e, -40 <= e <= 20
-}
-__device__ __forceinline__ void small_unit_flags(const float4* bodies, int64_t n, uint8_t* hflags) {
-    constexpr int U = 8;                               // loads in flight per lane (4096 bodies: 5 per lane)
-    const int nh = static_cast<int>(ceil_div<int64_t>(n, 32));
-    const int nw = static_cast<int>(blockDim.x >> 5), w = static_cast<int>(threadIdx.x >> 5);
-    const float* mass = reinterpret_cast<const float*>(bodies) + 3;
-    for (int h0 = w; h0 < nh; h0 += U * nw) {
-        float m[U], m0[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int h = h0 + u * nw, i = h * 32 + static_cast<int>(lane_id());
-            m[u] = m0[u] = 0.f;
-            if (h < nh) {
-                m0[u] = __ldcg(mass + 4 * ((h >> 1) * kChunkSmall));
-                m[u] = i < n ? __ldcg(mass + 4 * i) : m0[u];
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            const int h = h0 + u * nw;
-            const bool uni = __all_sync(0xffffffffu, m[u] == m0[u]) && unit_mass(m0[u]);
-            if (h < nh && lane_id() == 0) hflags[h] = uni ? 1 : 0;
-        }
-    }
-}
-// Bit c: chunk c of split s is mass-uniform (both its half chunks flagged).
-__device__ __forceinline__ uint32_t lane_unit_mask(const uint8_t* hflags, int s, int S, int L, int64_t n) {
-    uint32_t mask = 0;
-    if (s >= S) return 0;
-    const int nh = static_cast<int>(ceil_div<int64_t>(n, 32));
-    for (int c = 0; c < L / kChunkSmall; ++c) {
-        const int h = 2 * (s * (L / kChunkSmall) + c);
-        if (h >= nh) break;
-        const bool uni = hflags[h] != 0 && (h + 1 >= nh || hflags[h + 1] != 0);
-        mask |= static_cast<uint32_t>(uni) << c;
-    }
-    return mask;
-}
-
 // The lane's split partial for targets tg + 2p, tg + 2p + 1 (clamped to the last valid target),
 // then the butterfly over the warp's splits: lanes 2 (16 w) + p of each group's warp w end up with
 // the sum of splits 16 w .. 16 w + 15 (or the whole group when S2 <= 16), stored to wpart.
 // Every lane of the CTA's used warps calls it (lanes of split s >= S contribute zero).
-template <int U>
+template <int U, bool kKnown>
 __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLane& sl, bool active, int64_t tgt_first_src,
                                                int64_t tg, int64_t tcount, int L, int S, int S2, int64_t n, int chunk,
                                                float eps2, float4* wpart, uint64_t* tbar, uint32_t parity,
-                                               uint32_t umask) {
+                                               bool factor, uint32_t& known) {
     Interact<2, true> it;
     it.zero_all();
     LIME_WTRACE(0);
@@ -770,8 +748,8 @@ __device__ __forceinline__ void small_lane_sum(const float4* src, const SmallLan
     __syncwarp();
     if (active && sl.s < S) {
         const int64_t j0 = static_cast<int64_t>(sl.s) * L;
-        split_sum<U>(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
-                  eps2, umask);
+        split_sum<U, kKnown>(it, src + static_cast<int64_t>(sl.s) * (L + 1), static_cast<int>(mn<int64_t>(n, j0 + L) - j0), chunk,
+                  eps2, factor, known);
     }
     float4 a0 = it.result(0), a1 = it.result(1);
     const int seg = S2 < kWarpSplits ? kGroupPairs * S2 : 32;   // lanes of one group within this warp
@@ -840,10 +818,11 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) force_small_kernel(const 
     const int ct = static_cast<int>(threadIdx.x);
     // rounds of `slots` groups (one round by default); every lane calls small_lane_sum (whole warps
     // take part in its butterfly), lanes beyond the round's groups inactive
+    uint32_t known = 0;                                // the lane's verified factored chunks (split_sum)
     for (int64_t r0 = gb; r0 < ge; r0 += slots) {
         const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
-        small_lane_sum<kSmallUnroll>(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
-                       a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0, 0u);
+        small_lane_sum<kSmallUnroll, false>(src, sl, sl.gslot < ng, a.tgt_begin, (r0 + sl.gslot) * kGroupTargets, a.tgt_count, a.L, a.S,
+                       a.S2, a.n_src, a.chunk, a.eps2, wpart, a.tma ? tbar : nullptr, 0, a.eps2 >= 1e-20f, known);
         __syncthreads();
         const int64_t t = r0 * kGroupTargets + ct;
         if (ct < ng * kGroupTargets && t < a.tgt_count) {
@@ -925,7 +904,6 @@ struct SimArgs {
     int gq, gr;          // groups / grid, groups % grid (group_begin)
     float eps2, dt;
     int tma, rows;
-    int factor;          // eps2 >= 1e-20: factored mass-uniform chunks allowed (see small_unit_flags)
 };
 
 __device__ __forceinline__ void grid_barrier(unsigned* arrivals, unsigned target) {
@@ -949,7 +927,6 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
     float4* src = reinterpret_cast<float4*>(small_smem);                                     // [S][L + 1]
     float4* wpart = reinterpret_cast<float4*>(small_smem + small_src_bytes(a.rows, a.L));   // [slots][blocks][4]
     __shared__ __align__(8) uint64_t tbar[kMaxStageCopies];
-    __shared__ uint8_t hflags[kMaxHalfChunks];
     if (a.tma) {
         if (threadIdx.x < static_cast<unsigned>(kMaxStageCopies)) mbar_init(&tbar[threadIdx.x], 1);
         fence_mbar_init();
@@ -961,7 +938,7 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
     const int slots = static_cast<int>(blockDim.x) >> (__ffs(kGroupPairs * a.S2) - 1);   // a power of two
     const int ct = static_cast<int>(threadIdx.x);      // combine thread: one target of the round's groups
     unsigned barrier_target = 0;
-    uint32_t umask = 0;                                // the lane's factored chunks (masses never change: step 0)
+    uint32_t known = 0;                                // verified factored chunks: masses never change
 
     for (int32_t k = 0; k < a.steps; ++k) {
         const float4* cur = (k & 1) ? a.pos_alt : a.pos;
@@ -981,11 +958,6 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             stage_all<true>(src, cur, a.n, a.L);   // what every CTA wrote in the previous step (L2)
             __syncthreads();
         }
-        if (k == 0) {
-            small_unit_flags(a.pos, a.n, hflags);      // step 0 reads pos: nothing has written it yet
-            __syncthreads();
-            umask = a.factor ? lane_unit_mask(hflags, sl.s, a.S, a.L, a.n) : 0u;
-        }
         LIME_TRACE_AT(k, 6);
         for (int64_t r0 = gb; r0 < ge; r0 += slots) {
             const int ng = static_cast<int>(mn<int64_t>(slots, ge - r0));
@@ -993,8 +965,9 @@ __global__ void __launch_bounds__(kSmallMaxThreads, 1) simulate_small_kernel(con
             const bool owner = ct < ng * kGroupTargets && t < a.n;
             float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
             if (owner) v = a.vel[t];                   // issued before the force work: latency hidden
-            small_lane_sum<kSimUnroll>(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
-                           a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1), umask);
+            small_lane_sum<kSimUnroll, true>(src, sl, sl.gslot < ng, 0, (r0 + sl.gslot) * kGroupTargets, a.n, a.L, a.S, a.S2, a.n, a.chunk,
+                           a.eps2, wpart, a.tma ? tbar : nullptr, static_cast<uint32_t>(k & 1), a.eps2 >= 1e-20f,
+                           known);
             LIME_TRACE_AT(k, 4);
             __syncthreads();
             LIME_TRACE_AT(k, 1);
@@ -1089,7 +1062,6 @@ cudaError_t launch_simulate(float4* pos, float4* vel, int64_t n, int32_t steps, 
     a.dt = dt;
     a.tma = p.tma;
     a.rows = p.rows;
-    a.factor = (eps2 >= 1e-20f && LIME_SIM_FACTOR) ? 1 : 0;
     CUtensorMap map_pos, map_alt;
     std::memset(&map_pos, 0, sizeof map_pos);
     std::memset(&map_alt, 0, sizeof map_alt);

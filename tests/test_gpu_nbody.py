@@ -381,11 +381,12 @@ def test_tma_staged_sizes_match_general_kernel(lime, n):
     assert torch.equal(pos, pe) and torch.equal(vel, ve)
 
 
-# ------------------------------ R11 at the small sizes: factored power-of-two chunks (persistent simulation)
+# ------------------------------ R11 at the small sizes: factored power-of-two chunks (every small kernel)
 def _mixed_chunk_bodies(n, seed):
-    """Chunk 0 (and every chunk not listed) mass 2^-12; chunk 1 random masses; chunk 2 one body off
-    by one ulp; chunk 3 massless; chunk 4 equal but not a power of two (1/3000); chunk 5 equal 2^-41
-    (outside the factored range); the ragged last chunk 2^3."""
+    """Chunk 0 (and every chunk not listed) mass 2^-12; chunk 1 random masses; chunk 2 one body
+    (not first, middle or last: the kernels' prediction says "factored") off by one ulp; chunk 3
+    massless; chunk 4 equal but not a power of two (1/3000); chunk 5 equal 2^-41 (outside the
+    factored range); the ragged last chunk 2^3."""
     b = inputs.nbody_bodies(n, seed=seed)
     b[:, 3] = np.float32(2.0 ** -12)
     rng = np.random.default_rng(seed)
@@ -400,30 +401,45 @@ def _mixed_chunk_bodies(n, seed):
 
 
 @pytest.mark.parametrize("n", [400, 4096, 4160, 5000, 8192])
-def test_simulate_factored_chunks_bit_identical(lime, n):
-    # simulate_small_kernel sums chunks of equal power-of-two masses in the factored (11-op) form;
-    # scaling by a power of two is exact, so it must still equal eager per-body steps bit for bit,
-    # and the oracle within tolerance
+def test_small_factored_chunks_bit_identical(lime, n):
+    # the small kernels sum chunks of equal power-of-two masses in the factored (11-op) form, which
+    # has the per-body form's bits: the in-CTA map, the general kernel (launch overrides, per-body
+    # form), the staging-ablation variants, shards, the fused step and the persistent simulation
+    # must all agree bit for bit, and with the oracle within tolerance
     b_np = _mixed_chunk_bodies(n, 400 + n)
     b = _dev(b_np)
+    full = lime.map_nbody(b, float(EPS2))
+    ref, mag = oracle.nbody_accel(b_np, EPS2, with_mag=True)
+    assert nbody_rel_err(full.cpu().numpy(), ref, mag).max() <= NBODY_RTOL
+    for block, R in [(128, 1), (256, 2), (512, 4)]:
+        with lime.launch_override(block_threads=block, per_thread=R):
+            assert torch.equal(lime.map_nbody(b, float(EPS2)), full), (block, R)
+    for v in range(1, 7 if n <= 4096 else 6):              # variant 6: constant memory, <= 4096 bodies
+        with lime.nbody_variant(v):
+            assert torch.equal(lime.map_nbody(b, float(EPS2)), full), v
+    begin, count = n // 3, n // 2
+    assert torch.equal(lime.map_nbody(b, float(EPS2), begin, count), full[begin:begin + count])
     v0 = (inputs.nbody_bodies(n, seed=401 + n) * np.float32(0.05)).astype(np.float32)
     v0[:, 3] = 0
+    v = _dev(v0)
+    p_new = lime.map_nbody_step(b, float(EPS2), 1e-3, v)
+    p_ref, v_ref = b.clone(), _dev(v0)
+    lime.map_nbody_integrate(p_ref, v_ref, full, 1e-3)
+    assert torch.equal(p_new, p_ref) and torch.equal(v, v_ref)
     pos, vel = b.clone(), _dev(v0)
     lime.nbody_simulate(pos, vel, 4, float(EPS2), 1e-3)
     pe, ve = b.clone(), _dev(v0)
     _eager_steps(lime, pe, ve, 4)
     assert torch.equal(pos, pe) and torch.equal(vel, ve)
-    # one step from rest against the oracle: v1 = a dt (dt = 2^-10, exact scaling)
-    p1, v1 = b.clone(), torch.zeros_like(b)
-    lime.nbody_simulate(p1, v1, 1, float(EPS2), 2.0 ** -10)
-    ref, mag = oracle.nbody_accel(b_np, EPS2, with_mag=True)
-    assert nbody_rel_err(v1.cpu().numpy() * 1024.0, ref, mag).max() <= NBODY_RTOL
 
 
-def test_simulate_factored_needs_softening(lime):
+def test_small_factored_needs_softening(lime):
     # eps^2 < 1e-20 turns the factored form off (it bounds R^-3); still bit-identical
     n = 4096
     b = _dev(_mixed_chunk_bodies(n, 9))
+    full = lime.map_nbody(b, 1e-22)
+    with lime.launch_override(block_threads=256, per_thread=2):
+        assert torch.equal(lime.map_nbody(b, 1e-22), full)
     pos, vel = b.clone(), torch.zeros_like(b)
     lime.nbody_simulate(pos, vel, 2, 1e-22, 1e-3)
     pe, ve = b.clone(), torch.zeros_like(b)
