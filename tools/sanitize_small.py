@@ -38,6 +38,12 @@ def main():
     lime.map_nbody(e8, 1e-4, 0, 257)
     pt, vv = t.clone(), torch.zeros_like(t)
     lime.nbody_simulate(pt, vv, 3, 1e-4, 1e-3)
+    # round 2: factored power-of-two chunks -- predicted and verified (chunk 1 one mass off: the
+    # per-body redo), cached across steps in the persistent kernel
+    mx = t.clone()
+    mx[64 + 7, 3] *= 2.0
+    lime.map_nbody(mx, 1e-4)
+    lime.nbody_simulate(mx.clone(), torch.zeros_like(mx), 3, 1e-4, 1e-3)
     S, X, T = (torch.from_numpy(a).to(dev) for a in inputs.blackscholes_options(4099, seed=3))
     lime.map_blackscholes(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
     lime.map_reduce_blackscholes_sum(S, X, T, inputs.BS_R, inputs.BS_SIGMA)
