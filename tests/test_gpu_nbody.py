@@ -445,3 +445,27 @@ def test_small_factored_needs_softening(lime):
     pe, ve = b.clone(), torch.zeros_like(b)
     _eager_steps(lime, pe, ve, 2, eps2=1e-22)
     assert torch.equal(pos, pe) and torch.equal(vel, ve)
+
+
+def test_small_factored_edge_masses_bitwise(lime):
+    # range ends of the factored form (2^-40 and 2^20 factored; 2^-41, 2^21, subnormal, -0, inf and
+    # NaN masses not) -- the in-CTA kernel must match the general per-body kernel bit for bit
+    # (compared as raw words, so NaN results compare too)
+    n = 1024
+    b = inputs.nbody_bodies(n, seed=77)
+    b[:, 3] = np.float32(2.0 ** -12)
+    masses = [2.0 ** -40, 2.0 ** 20, 2.0 ** -41, 2.0 ** 21, 2.0 ** -130, -0.0, 1.0]
+    for c, m in enumerate(masses):
+        b[64 * (c + 1):64 * (c + 2), 3] = np.float32(m)
+    b[64 * 9 + 5, 3] = np.inf
+    b[64 * 10 + 9, 3] = np.nan
+    bd = _dev(b)
+    full = lime.map_nbody(bd, float(EPS2))
+    with lime.launch_override(block_threads=128, per_thread=2):
+        gen = lime.map_nbody(bd, float(EPS2))
+    assert torch.equal(full.view(torch.int32), gen.view(torch.int32))
+    pos, vel = bd.clone(), torch.zeros_like(bd)
+    lime.nbody_simulate(pos, vel, 2, float(EPS2), 1e-3)
+    pe, ve = bd.clone(), torch.zeros_like(bd)
+    _eager_steps(lime, pe, ve, 2)
+    assert torch.equal(pos.view(torch.int32), pe.view(torch.int32)) and torch.equal(vel.view(torch.int32), ve.view(torch.int32))
