@@ -11,9 +11,10 @@
 // The element function is written for B200's ridge point: 6 MUFU per option,
 // two options per packed FFMA2/FMUL2 instruction. Savings vs the textbook evaluation:
 //   * 1/(sigma sqrt T) = rsqrt(T) / sigma  (one MUFU.RSQ gives both sqrt T and its inverse)
-//   * ln(S/X) = (lg2 S - lg2 X) ln 2
+//   * ln(S/X) = lg2(S rcp X) ln 2 (map; the fused sums use (lg2 S - lg2 X) ln 2)
 //   * K phi(d2) = S phi(d1) (exact identity, K = X e^{-rT}) -> one exponential serves both
-//     normal-CDF tails (Abramowitz & Stegun 26.2.17, |err| < 7.5e-8).
+//     normal-CDF tails (map: a degree-7 Mills-ratio polynomial, |err| < 5e-10; fused sums:
+//     Abramowitz & Stegun 26.2.17, |err| < 7.5e-8).
 // The map evaluates call and put per option (price2, ~48 FP32 lane-ops); the fused sums use
 // price2_wu (~34 lane-ops, no per-option selects), which sums w and u with call = w + u/2 and
 // put = w - u/2.
@@ -49,15 +50,23 @@ __device__ __forceinline__ float as_poly(float k) {
 }
 
 // Two options per call, packed (FFMA2/FMUL2/FADD2 carry both; MUFU ops are per lane).
-// Per option: 6 MUFU (rsqrt T, lg2 S, lg2 X, ex2 -rT, ex2 -d1^2/2, and ONE rcp shared by the two
-// Abramowitz-Stegun k's: k1 = D2/(D1 D2), k2 = D1/(D1 D2)).
+// Per option: 6 MUFU (rsqrt T, rcp X + lg2 S/X, ex2 -rT, ex2 -d1^2/2, and ONE rcp shared by the two
+// CND k's: k1 = D2/(D1 D2), k2 = D1/(D1 D2)).
 struct P2 { float2 call, put; };
 
-__device__ __forceinline__ float2 as_poly2(float2 k) {
-    float2 p = fma2(k, bcast2(kAS_a5), bcast2(kAS_a4));
-    p = fma2(k, p, bcast2(kAS_a3));
-    p = fma2(k, p, bcast2(kAS_a2));
-    p = fma2(k, p, bcast2(kAS_a1));
+// Map element CND (round 2): N(-|x|) = phi(x) M(k), k = 1/(1 + p|x|), p = 0.318, M a degree-7
+// polynomial with M(0) = 0 fitted to the Mills ratio N(-x)/phi(x) by a weighted minimax (Lawson) fit
+// of phi(x) (M(k) - N(-x)/phi(x)) over x in [0, 40] (tools/fit_mills.py): max |dN| = 5.0e-10, against
+// 7.5e-8 for Abramowitz-Stegun 26.2.17 -- whose error times X <= 100 alone used up to 8.9e-6 of the
+// 1e-5 element tolerance (r = 0, sigma = 0.3: 1.03e-5 measured; profiles/experiments/bs_accuracy_r02.txt).
+constexpr float kM_p = 0.318f;
+__device__ __forceinline__ float2 mills7_2(float2 k) {
+    float2 p = fma2(k, bcast2(1.1605857361e-01f), bcast2(-6.2049898640e-01f));
+    p = fma2(k, p, bcast2(1.0789559974e+00f));
+    p = fma2(k, p, bcast2(-4.7603565775e-01f));
+    p = fma2(k, p, bcast2(5.7942646417e-01f));
+    p = fma2(k, p, bcast2(2.5091390071e-01f));
+    p = fma2(k, p, bcast2(3.2449384680e-01f));
     return mul2(k, p);
 }
 __device__ __forceinline__ float2 abs2(float2 v) { return make_float2(fabsf(v.x), fabsf(v.y)); }
@@ -67,23 +76,24 @@ __device__ __forceinline__ P2 price2(float2 S, float2 X, float2 T, const Consts&
     const float2 sqT = mul2(T, rsT);
     const float2 v = mul2(bcast2(c.sigma), sqT);                       // sigma sqrt T
     const float2 inv_v = mul2(rsT, bcast2(c.inv_sigma));               // 1 / (sigma sqrt T)
-    const float2 lg = sub2(make_float2(lg2_approx(S.x), lg2_approx(S.y)),
-                           make_float2(lg2_approx(X.x), lg2_approx(X.y)));
-    const float2 l = mul2(lg, bcast2(kLn2));                            // ln(S/X)
+    // ln(S/X) from one lg2 of the fp32 ratio (rcp + lg2: the same two MUFU as lg2 S - lg2 X, one
+    // rounding of S/X instead of two rounded logarithms of ~5 subtracted)
+    const float2 q = mul2(S, make_float2(rcp_approx(X.x), rcp_approx(X.y)));
+    const float2 l = mul2(make_float2(lg2_approx(q.x), lg2_approx(q.y)), bcast2(kLn2));   // ln(S/X)
     const float2 d1 = mul2(fma2(bcast2(c.r_plus_half_s2), T, l), inv_v);
     const float2 d2 = sub2(d1, v);
     const float2 er = mul2(bcast2(c.neg_r_log2e), T);
     const float2 K = mul2(X, make_float2(ex2_approx(er.x), ex2_approx(er.y)));   // X e^{-rT}
-    const float2 D1 = fma2(bcast2(kAS_p), abs2(d1), bcast2(1.f));
-    const float2 D2 = fma2(bcast2(kAS_p), abs2(d2), bcast2(1.f));
+    const float2 D1 = fma2(bcast2(kM_p), abs2(d1), bcast2(1.f));
+    const float2 D2 = fma2(bcast2(kM_p), abs2(d2), bcast2(1.f));
     const float2 DD = mul2(D1, D2);
     const float2 rr = make_float2(rcp_approx(DD.x), rcp_approx(DD.y));
     const float2 k1 = mul2(D2, rr);                                     // 1 / D1
     const float2 k2 = mul2(D1, rr);                                     // 1 / D2
     const float2 g = mul2(mul2(bcast2(kNegHalfLog2e), d1), d1);
     const float2 sphi = mul2(S, mul2(bcast2(kInvSqrt2Pi), make_float2(ex2_approx(g.x), ex2_approx(g.y))));
-    const float2 sq1 = mul2(sphi, as_poly2(k1));                       // S N(-|d1|)
-    const float2 kq2 = mul2(sphi, as_poly2(k2));                       // K N(-|d2|) = S phi(d1) poly(k2)
+    const float2 sq1 = mul2(sphi, mills7_2(k1));                       // S N(-|d1|)
+    const float2 kq2 = mul2(sphi, mills7_2(k2));                       // K N(-|d2|) = S phi(d1) poly(k2)
     const float2 s_m = sub2(S, sq1);                                    // S (1 - N(-|d1|))
     const float2 k_m = sub2(K, kq2);
     P2 r;
