@@ -111,3 +111,30 @@ def test_mandelbrot_regions_bit_exact(lime, x0, y0, span, max_iter):
     got = lime.map_mandelbrot(W, H, x0, y0, dx, dy, max_iter).cpu().numpy()
     ref = oracle.mandelbrot(W, H, 0, 1, H, x0, y0, dx, dy, max_iter)
     assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("dist", ["uniform", "two_clusters", "far_cube"])
+@pytest.mark.parametrize("eps2", [1e-12, 1e-4, 1.0])
+def test_nbody_f64_variants(lime, dist, eps2):
+    n = 3001
+    b = {"uniform": lambda n, s: inputs.nbody_bodies(n, seed=s), "two_clusters": two_clusters,
+         "far_cube": far_cube}[dist](n, 500).astype(np.float64)
+    acc = lime.map_nbody_f64(_dev(b), eps2).cpu().numpy()
+    ref, mag = oracle.nbody_accel_f64(b, eps2, with_mag=True)
+    assert nbody_rel_err(acc, ref, mag).max() <= 1e-12, (dist, eps2)
+
+
+def test_matmul_wide_dynamic_range(lime):
+    # bf16 operands with exponents spread over 2^-20 .. 2^20 (products over 2^-40 .. 2^40): the fp32
+    # tensor-core accumulation against sum_k |A_ik Bt_jk| (north_star 1e-3), ragged M/N/K
+    M, N, K = 300, 520, 264
+    A, Bt = inputs.matmul_operands(M, N, K, seed=600)
+    def spread(bits, seed):
+        e = (np.floor(_u(seed, 0, bits.size) * 41) - 20).reshape(bits.shape)
+        f = inputs.bf16_bits_to_f32(bits).astype(np.float64) * np.exp2(e)
+        return inputs._f32_to_bf16_bits(f.astype(np.float32))
+    A, Bt = spread(A, 601), spread(Bt, 602)
+    C = lime.map_matmul_bf16(_dev(A.view(np.int16)).view(torch.bfloat16), _dev(Bt.view(np.int16)).view(torch.bfloat16))
+    ref = oracle.matmul_bf16(A, Bt)
+    mag = np.abs(inputs.bf16_bits_to_f32(A)).astype(np.float64) @ np.abs(inputs.bf16_bits_to_f32(Bt)).astype(np.float64).T
+    assert (np.abs(C.cpu().numpy() - ref) / np.maximum(mag, 1e-300)).max() <= 1e-3
