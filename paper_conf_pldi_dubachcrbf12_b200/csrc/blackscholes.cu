@@ -257,23 +257,31 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
     }
     __syncthreads();
     if (!s_last) return;
-    // Last CTA: combine the CTA partials in index order (warp 0, fixed lane->CTA mapping).
+    // Last CTA: combine the CTA partials in a fixed order with every thread: thread t takes partials
+    // t, t + 256, ... (at most kMaxCtas / 256 = 5, all loads issued before the adds: one L2 round trip
+    // instead of the three of a one-warp loop), then the warp shuffle tree and the warps in order.
     __threadfence();
-    if (warp == 0) {
-        double bx = 0.0, by = 0.0;
-#pragma unroll 8
-        for (unsigned k = lane_id(); k < gridDim.x; k += 32) {   // unrolled: the L2 loads issue ahead of the adds
-            const double2 p = __ldcg(partial + k);
-            bx += p.x;
-            by += p.y;
-        }
-        bx = warp_sum(bx);
-        by = warp_sum(by);
-        if (lane_id() == 0) {
-            sums[0] = bx;
-            sums[1] = by;
-            *ticket = 0u;   // leave the workspace zeroed
-        }
+    constexpr int kPer = (red::kMaxCtas + 255) / 256;
+    double2 pv[kPer];
+#pragma unroll
+    for (int q = 0; q < kPer; ++q) {
+        const unsigned k = threadIdx.x + 256u * q;
+        pv[q] = k < gridDim.x ? __ldcg(partial + k) : make_double2(0.0, 0.0);
+    }
+    double bx = pv[0].x, by = pv[0].y;
+#pragma unroll
+    for (int q = 1; q < kPer; ++q) { bx += pv[q].x; by += pv[q].y; }
+    bx = warp_sum(bx);
+    by = warp_sum(by);
+    __syncthreads();                               // s_part[] was last read by thread 0 above
+    if (lane_id() == 0) s_part[warp] = make_double2(bx, by);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double2 b = s_part[0];
+        for (int k = 1; k < (blockDim.x >> 5); ++k) { b.x += s_part[k].x; b.y += s_part[k].y; }
+        sums[0] = b.x;
+        sums[1] = b.y;
+        *ticket = 0u;   // leave the workspace zeroed
     }
 }
 
