@@ -252,15 +252,17 @@ __global__ void __launch_bounds__(256, 4) map_reduce_kernel(const float* __restr
         double2 b = s_part[0];
         for (int k = 1; k < (blockDim.x >> 5); ++k) { b.x += s_part[k].x; b.y += s_part[k].y; }
         __stcg(partial + blockIdx.x, b);
-        __threadfence();
-        s_last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
+        // acq_rel ticket: releases this CTA's partial, and the last CTA's thread 0 acquires every
+        // other CTA's (the __syncthreads below extends the order to the combining threads)
+        unsigned prev;
+        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(ticket) : "memory");
+        s_last = (prev == gridDim.x - 1);
     }
     __syncthreads();
     if (!s_last) return;
     // Last CTA: combine the CTA partials in a fixed order with every thread: thread t takes partials
     // t, t + 256, ... (at most kMaxCtas / 256 = 5, all loads issued before the adds: one L2 round trip
     // instead of the three of a one-warp loop), then the warp shuffle tree and the warps in order.
-    __threadfence();
     constexpr int kPer = (red::kMaxCtas + 255) / 256;
     double2 pv[kPer];
 #pragma unroll
