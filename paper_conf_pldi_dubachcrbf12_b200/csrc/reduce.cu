@@ -157,30 +157,20 @@ __global__ void __launch_bounds__(256) reduce_kernel(const T* __restrict__ x, in
     __syncthreads();
     if (!s_last) return;
     __threadfence();
-    // fixed order (deterministic for a given grid), every thread: thread t folds partials t, t + 256,
-    // ... (at most kMaxCtas / 256, all loads issued before the folds -- one L2 round trip instead of
-    // the three of a one-warp loop), then the xor-shuffle tree and the warps in index order
-    constexpr int kPer = (kMaxCtas + 255) / 256;
-    A pv[kPer];
-#pragma unroll
-    for (int q = 0; q < kPer; ++q) {
-        const unsigned k = threadIdx.x + 256u * q;
-        pv[q] = k < gridDim.x ? ldcg_acc(partial + k) : P::id();
-    }
-    A b = pv[0];
-#pragma unroll
-    for (int q = 1; q < kPer; ++q) b = P::comb(b, pv[q]);
-    b = warp_reduce<P>(b);
-    if (lane_id() == 0) s_warp[warp] = b;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        b = s_warp[0];
-        for (int w = 1; w < (blockDim.x >> 5); ++w) b = P::comb(b, s_warp[w]);
-        if constexpr (OP != kSum && std::is_floating_point<T>::value) {
-            if (n == 0) b = (OP == kMin) ? static_cast<A>(INFINITY) : static_cast<A>(-INFINITY);  // R9
+    if (warp == 0) {
+        // fixed order (deterministic for a given grid): lane l folds partials l, l+32, ... in index
+        // order, then the fixed xor-shuffle tree combines the 32 lane values
+        A b = P::id();
+#pragma unroll 8
+        for (unsigned k = lane_id(); k < gridDim.x; k += 32) b = P::comb(b, ldcg_acc(partial + k));   // loads issue ahead
+        b = warp_reduce<P>(b);
+        if (lane_id() == 0) {
+            if constexpr (OP != kSum && std::is_floating_point<T>::value) {
+                if (n == 0) b = (OP == kMin) ? static_cast<A>(INFINITY) : static_cast<A>(-INFINITY);  // R9
+            }
+            *out = static_cast<T>(b);
+            *ticket = 0u;
         }
-        *out = static_cast<T>(b);
-        *ticket = 0u;
     }
 }
 
