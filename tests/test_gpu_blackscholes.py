@@ -74,3 +74,16 @@ def test_fused_single_option_tails(lime, k):
     sc, sp = oracle.blackscholes_sums(s, x, t, R, SIG)
     assert abs(sums[0] - sc) <= BS_TOL * max(abs(sc), 8.0)       # per option: 1e-5 * max(|price|, 1)
     assert abs(sums[1] - sp) <= BS_TOL * max(abs(sp), 8.0)
+
+
+@pytest.mark.parametrize("grid", [1, 7, 148, 255, 256, 257, 1184])
+def test_fused_sums_launch_configs(lime, grid):
+    # the last CTA combines every CTA partial (up to kMaxCtas = 1184: five per thread)
+    n = (1 << 20) + 3
+    S, X, T = inputs.blackscholes_options(n, seed=9)
+    sc, sp = oracle.blackscholes_sums(S, X, T, R, SIG)
+    with lime.launch_override(grid_ctas=grid):
+        sums = lime.map_reduce_blackscholes_sum(_dev(S), _dev(X), _dev(T), float(R), float(SIG)).cpu().numpy()
+        again = lime.map_reduce_blackscholes_sum(_dev(S), _dev(X), _dev(T), float(R), float(SIG)).cpu().numpy()
+    assert abs(sums[0] - sc) <= BS_TOL * abs(sc) and abs(sums[1] - sp) <= BS_TOL * abs(sp), grid
+    assert np.array_equal(sums, again)
