@@ -22,10 +22,15 @@ namespace nbody {
 // Two-level accumulation (part of the result's definition, a function of n_src only): sources are
 // cut into chunks of chunk_len(n_src) bodies whose partials are added in order into one of
 // splits(n_src) split partials, added in split order. Small problems (n_src <= kSmallMaxSources)
-// use 128-body chunks and up to 32 splits (twice the warps for the latency-bound sizes), larger
-// ones 256-body chunks and up to 16 splits.
+// use 64-body chunks and up to 64 splits (whole warps per SMSP for the latency-bound sizes), larger
+// ones 256-body chunks and up to 32 splits (r02: 16 -> 32 -- the 2^20 launch is 8192 -> 16384 CTAs of
+// one SM each, so its last wave idles 44 instead of 96 SMs: 377.7 -> 373.4 ms, same-call A/B).
 constexpr int kChunk = 256;
-constexpr int kMaxSplits = 16;
+#ifndef LIME_MAX_SPLITS              // compile-time A/B override (tools/); the default is the product
+#define LIME_MAX_SPLITS 32
+#endif
+constexpr int kMaxSplits = LIME_MAX_SPLITS;
+constexpr int kMaxSplitsF64 = 16;   // the fp64 map's own rule (chunks_per_split_fixed / splits_fixed)
 #ifndef LIME_CHUNK_SMALL            // compile-time A/B overrides (tools/); the defaults are the product
 #define LIME_CHUNK_SMALL 64
 #endif
@@ -38,7 +43,7 @@ constexpr int64_t kSmallMaxSources = 8192;
 int chunk_len(int64_t n_src);
 int64_t chunks_per_split(int64_t n_src);
 int splits(int64_t n_src);
-int64_t chunks_per_split_fixed(int64_t n_src);   // 256-body chunks, <= 16 splits (fp64 map)
+int64_t chunks_per_split_fixed(int64_t n_src);   // 256-body chunks, <= kMaxSplitsF64 splits (fp64 map)
 int splits_fixed(int64_t n_src);
 size_t workspace_bytes(int64_t n_src, int64_t tgt_count);
 cudaError_t launch_force(const float4* bodies, int64_t n_src, int64_t tgt_begin, int64_t tgt_count,

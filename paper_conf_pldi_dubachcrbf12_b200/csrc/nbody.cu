@@ -66,8 +66,8 @@ static int splits_rule(int64_t n_src, int chunk, int maxs) {
 }
 int64_t chunks_per_split(int64_t n_src) { return cps_rule(n_src, chunk_len(n_src), max_splits(n_src)); }
 int splits(int64_t n_src) { return splits_rule(n_src, chunk_len(n_src), max_splits(n_src)); }
-int64_t chunks_per_split_fixed(int64_t n_src) { return cps_rule(n_src, kChunk, kMaxSplits); }
-int splits_fixed(int64_t n_src) { return splits_rule(n_src, kChunk, kMaxSplits); }
+int64_t chunks_per_split_fixed(int64_t n_src) { return cps_rule(n_src, kChunk, kMaxSplitsF64); }
+int splits_fixed(int64_t n_src) { return splits_rule(n_src, kChunk, kMaxSplitsF64); }
 
 // workspace: [counters: one u32 per 128-target tile, padded to 256 B]
 //            [chunk flags: one byte per 256-body source chunk when n_src > kSmallMaxSources, padded to 256 B]

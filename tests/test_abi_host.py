@@ -143,14 +143,14 @@ def test_no_device_reports_unsupported(L):
 
 def test_workspace_queries_and_split_rule(L):
     # splits depend on n_src only (deterministic order across shards/launches)
-    # n_src <= 8192: 64-body chunks, <= 64 splits; larger: 256-body chunks, <= 16 splits
+    # n_src <= 8192: 64-body chunks, <= 64 splits; larger: 256-body chunks, <= 32 splits
     assert L.lime_nbody_splits(1) == 1 and L.lime_nbody_splits(64) == 1
     assert L.lime_nbody_splits(65) == 2 and L.lime_nbody_splits(129) == 3
     assert L.lime_nbody_splits(4096) == 64
     assert L.lime_nbody_splits(4097) == 33          # 65 chunks, 2 per split
     assert L.lime_nbody_splits(8192) == 64          # 128 chunks, 2 per split
-    assert L.lime_nbody_splits(8193) == 11          # 33 chunks of 256, 3 per split
-    assert L.lime_nbody_splits(1 << 20) == 16
-    assert L.lime_map_nbody_workspace_bytes(1 << 20, 1 << 17) >= 16 * (1 << 17) * 16
+    assert L.lime_nbody_splits(8193) == 17          # 33 chunks of 256, 2 per split
+    assert L.lime_nbody_splits(1 << 20) == 32
+    assert L.lime_map_nbody_workspace_bytes(1 << 20, 1 << 17) >= 32 * (1 << 17) * 16
     assert L.lime_reduce_workspace_bytes() >= 256
     assert L.lime_mandelbrot_workspace_bytes() >= 8
