@@ -103,10 +103,12 @@ void lime_set_launch_override(int grid_ctas, int block_threads, int per_thread);
  *   eps2    Plummer softening, finite and > 0 (eps2 <= 0 makes the self term 0/0).
  *   0 <= tgt_begin, 0 <= tgt_count, tgt_begin + tgt_count <= n_src.
  * Summation order (deterministic, independent of launch config and of the
- * target shard): sources are cut into chunks (128 bodies when n_src <= 8192,
+ * target shard): sources are cut into chunks (64 bodies when n_src <= 8192,
  * else 256); each chunk is summed in j order into a chunk partial; chunk
- * partials are added in order into one of
- * S = nbody_splits(n_src) split partials; split partials are added in s order.
+ * partials are added in order into one of S = nbody_splits(n_src) split
+ * partials (S <= 64 when n_src <= 8192, else <= 32); split partials are added
+ * as a pairwise tree over next_pow2(S) leaves when n_src <= 8192, else in s
+ * order (R11).
  * Mass-uniform splits (n_src > 8192; R11): when every body of a
  * split has the same mass m (bitwise-equal floats), each chunk partial is
  * sum_j (p_j - p_i) / R^3 and is added as m * partial (exact algebra, one fewer
