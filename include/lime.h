@@ -219,7 +219,7 @@ lime_status lime_map_blackscholes(const float *S, const float *X, const float *T
 /* Fused map+reduce (`!` over `@` without materialising the map, L160-163,
  * L188-189; R6): sums[0] = sum_i call[i], sums[1] = sum_i put[i]
  * (device double[2]), accumulated in fp64 from the warp level up (per-thread
- * partials fp32), CTA partials combined in fixed index order by the last CTA
+ * partials fp32), CTA partials combined in a fixed order by the last CTA
  * (deterministic for a given launch configuration). The element is the same
  * closed form rearranged for summation: with A = S N(d1) - S/2 and
  * B = K N(d2) - K/2 (K = X e^{-rT}), call = (A - B) + (S - K)/2 and

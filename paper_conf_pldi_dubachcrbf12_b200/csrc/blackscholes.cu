@@ -4,7 +4,8 @@
 // streaming loads of the SoA operands (ld.global.nc.L1::no_allocate, PAPER.md L267-275
 // vectorisation of read-only arrays) and evict-first 128-bit stores. A8: the fused
 // variant never writes call/put; fp32 partials per thread -> fp64 from the warp up -> CTA ->
-// last CTA combines CTA partials in index order. Both kernels are launched with programmatic
+// the last CTA (acq_rel ticket) combines the CTA partials in a fixed order with all its threads.
+// Both kernels are launched with programmatic
 // dependent launch (common.cuh pdl_enter/launch_pdl), so back-to-back launches overlap the
 // next grid's launch with this one's drain.
 //
